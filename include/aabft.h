@@ -1,0 +1,214 @@
+/*
+ * aabft.h -- C ABI of the B200-native (sm_100a) A-ABFT hot path.
+ *
+ * A-ABFT: Braun, Halder, Wunderlich, "A-ABFT: Autonomous Algorithm-Based Fault Tolerance
+ * for Matrix Multiplications on Graphics Processing Units", DSN 2014.  "P:Lnn" cites line
+ * nn of the paper text; section / equation / algorithm given beside it.
+ *
+ * The path (§V):
+ *   1. aabft_encode   -- partitioned checksums of A (column checksums per BS rows, Eq 1) and
+ *                        of B (row checksums per BS columns, Eq 2) fused with the top-p
+ *                        largest |values| of every row of A / column of B and of every
+ *                        checksum row / column (Alg 1; step 3 global reduction)
+ *   2. aabft_gemm     -- checksum-augmented product C_fc = A_cc . B_rc (Eq 3): C, the carried
+ *                        column checksums Ccol = Acs.B and row checksums Crow = A.Bcs
+ *   3. aabft_check    -- bound (§IV, Eq 28 / P:L287, upper bound y §IV-E), reference sums
+ *                        (Eq 4), comparison (Eq 6) and 3-class classification
+ *   4. aabft_correct  -- locate a single critical error at the intersection of the
+ *                        mismatching row and column and correct it (Alg 2 output,
+ *                        P:L385)
+ * plus aabft_bound (the bound alone, §IV-E last paragraph P:L307) and aabft_gemm_plain (the
+ * unprotected GEMM of the same kernel family; the overhead denominator).
+ *
+ * Conventions (all entry points):
+ *  - Every matrix is ROW-MAJOR; "ld" is the row pitch in ELEMENTS.  All array pointers are
+ *    DEVICE pointers unless the name ends in _host.  The caller owns all memory: the library
+ *    never allocates, frees or synchronises (except aabft_protected_gemm_host, which
+ *    synchronises its stream before returning because it writes host memory).
+ *  - Every call is asynchronous on `stream` (a cudaStream_t passed as void*; NULL = legacy
+ *    default stream).  AABFT_OK means "validated and enqueued".
+ *  - Parameter checks run before any launch and return AABFT_EINVAL with a message in
+ *    aabft_last_error().  Launch failures return AABFT_ECUDA.  A device that is not sm_100
+ *    returns AABFT_EUNSUPPORTED.  No C++ exception crosses this ABI.
+ *  - Inputs must be finite; non-finite RESULTS are always classified CRITICAL (reading R9).
+ *  - Thread safety: calls are safe concurrently on distinct streams and buffers.
+ */
+#ifndef AABFT_H
+#define AABFT_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  AABFT_OK = 0,
+  AABFT_EINVAL = 1,        /* bad argument (dimension, ld, alignment, NULL, range) */
+  AABFT_EUNSUPPORTED = 2,  /* not an sm_100 device */
+  AABFT_ECUDA = 3,         /* CUDA launch / runtime error (message in aabft_last_error) */
+  AABFT_EWORKSPACE = 4,    /* workspace NULL or too small */
+  AABFT_EINTERNAL = 5
+} aabft_status;
+
+typedef enum { AABFT_F64 = 0, AABFT_F32 = 1 } aabft_dtype;
+
+/* Problem description.  C[M x N] = A[M x K] . B[K x N].
+ *  bs        checksum block size BS (partitioned encoding, P:L91 ref [20]); power of two in
+ *            [8, 256]; M % bs == 0 and N % bs == 0 (the caller zero-pads: "padded matrix A",
+ *            Alg 1; reading R20).  K is free (>= 1).
+ *  p         numMax, the number of largest |values| per vector; 1..8, p <= K.
+ *  omega     confidence scale of Eq 7; the paper uses 3.
+ *  t         eps_M = 2^-t; 0 selects 52 (F64) / 23 (F32) (reading R1).
+ *  fma_model 1: sigma of Eq 28 (FMA hardware, §IV-D) -- the default;
+ *            0: sigma of P:L287 plus |EV_Prod| of Eq 43 (separately rounded products). */
+typedef struct {
+  int32_t dtype;  /* aabft_dtype: element type of A, B, C, Acs, Bcs, Ccol, Crow */
+  int32_t bs;
+  int64_t M, N, K;
+  int32_t p;
+  int32_t t;
+  double omega;
+  int32_t fma_model;
+  int32_t reserved;
+} aabft_config;
+
+/* Output of aabft_encode.  Acs: (M/bs) x K, ld_acs >= K.  Bcs: K x (N/bs), ld_bcs >= N/bs.
+ * topA_val/topA_idx: (M + M/bs) x p -- data rows 0..M-1, then checksum rows; |value|
+ *   (as double) in descending order, ties to the lowest index; idx = column k.
+ * topB_val/topB_idx: (N + N/bs) x p -- data columns, then checksum columns; idx = row k. */
+typedef struct {
+  void *Acs;
+  int64_t ld_acs;
+  void *Bcs;
+  int64_t ld_bcs;
+  double *topA_val;
+  int32_t *topA_idx;
+  double *topB_val;
+  int32_t *topB_idx;
+} aabft_encoded;
+
+/* Output of aabft_gemm.  C: M x N (ldc >= N); Ccol: (M/bs) x N (ld_ccol >= N) carried column
+ * checksums c_{m+1,j} per block-row; Crow: M x (N/bs) (ld_crow >= N/bs) carried row
+ * checksums c_{i,q+1} per block-column (Eq 3 with partitioned encoding; corner not formed,
+ * reading R17). */
+typedef struct {
+  void *C;
+  int64_t ldc;
+  void *Ccol;
+  int64_t ld_ccol;
+  void *Crow;
+  int64_t ld_crow;
+} aabft_product;
+
+/* Per-block (BS x BS sub-matrix of C, "one threadblock for each submatrix of C")
+ * report, row-major over blocks: report[I * (N/bs) + J]. */
+enum {
+  AABFT_BLK_CLEAN = 0,          /* no critical check */
+  AABFT_BLK_CORRECTED = 1,      /* one critical row x one critical column, corrected */
+  AABFT_BLK_CHECKSUM_ONLY = 2,  /* only row checks or only column checks tripped: the
+                                   carried checksum itself is faulty, data untouched */
+  AABFT_BLK_UNCORRECTABLE = 3,  /* several rows and columns, or correction did not verify */
+  AABFT_BLK_SINGLE = 4          /* located by aabft_check, awaiting aabft_correct */
+};
+typedef struct {
+  uint8_t status;      /* AABFT_BLK_* */
+  uint8_t worst_class; /* 0 rounding, 1 tolerable, 2 critical (reading R10) */
+  uint16_t n_bad_rows; /* critical row checks in the block */
+  uint16_t n_bad_cols; /* critical column checks in the block */
+  uint16_t reserved;
+  int32_t row, col;    /* global (i, j) of the located element, else -1 */
+  float max_ratio;     /* max |d| / eps over the block's 2*bs checks (inf if eps = 0 < |d|) */
+} aabft_block_report;  /* 20 bytes */
+
+/* Device-side counters, reducible with a SUM all-reduce (n) and a MAX all-reduce
+ * (max_ratio): n = {blocks, clean, corrected, checksum_only, uncorrectable,
+ * checks_rounding, checks_tolerable, checks_critical}. */
+typedef struct {
+  int64_t n[8];
+  double max_ratio;
+} aabft_counts;
+
+/* Fault descriptor for injection campaigns (Alg 3).
+ * (row, col) are C_fc coordinates: row in [M, M + M/bs) hits Ccol row row-M;
+ * col in [N, N + N/bs) hits Crow column col-N.
+ *  site 0: XOR xor_mask into the stored result ("errorVecAdd2")
+ *  site 1: XOR xor_mask into the accumulator after the k-tile that contains k_step
+ *          ("errorVecAdd1" at k-tile granularity; products inside the DMMA unit
+ *          are not addressable)
+ *  site 2: add `add` to the stored result (magnitude sweep) */
+typedef struct {
+  int64_t row, col;
+  int32_t site;
+  int32_t reserved;
+  int64_t k_step;
+  uint64_t xor_mask;
+  double add;
+} aabft_fault; /* 48 bytes */
+
+/* Bytes of device workspace needed by aabft_encode / aabft_gemm / aabft_check (one buffer
+ * serves all three; 256-byte aligned).  Returns 0 on an invalid config. */
+size_t aabft_workspace_bytes(const aabft_config *cfg);
+
+/* Step 1 (Alg 1).  A (lda >= K) or B (ldb >= N) may be NULL to encode only the
+ * other; the corresponding outputs are then untouched.  Checksums are summed sequentially
+ * in ascending order in the working precision, so Acs/Bcs, top-p values and hence every
+ * bound are bit-identical to the definition (reading R11). */
+aabft_status aabft_encode(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
+                          int64_t ldb, const aabft_encoded *out, void *ws, size_t ws_bytes,
+                          void *stream);
+
+/* Bound alone (§IV-E): eps for every carried checksum element.
+ * eps_col: (M/bs) x N dense, eps_row: M x (N/bs) dense (either may be NULL); sig_* likewise.
+ * eps = omega * sqrt(F(K)) * y * 2^-t (+ K/3 * 2^-2t * y when fma_model = 0). */
+aabft_status aabft_bound(const aabft_config *cfg, const aabft_encoded *enc, double *eps_col,
+                         double *sig_col, double *eps_row, double *sig_row, void *stream);
+
+/* Step 2 (Eq 3).  FP64: DMMA (mma.sync .f64) tensor-core tiles fed by TMA;
+ * FP32: FFMA SIMT tiles (no TF32: it would change the rounding model, north_star).
+ * faults: DEVICE array of nfaults aabft_fault (NULL / 0 = none). */
+aabft_status aabft_gemm(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
+                        int64_t ldb, const aabft_encoded *enc, const aabft_product *out,
+                        const aabft_fault *faults, int32_t nfaults, void *ws, size_t ws_bytes,
+                        void *stream);
+
+/* Unprotected C = A.B with the same kernel family (overhead denominator). */
+aabft_status aabft_gemm_plain(const aabft_config *cfg, const void *A, int64_t lda,
+                              const void *B, int64_t ldb, void *C, int64_t ldc, void *stream);
+
+/* Step 3 (Alg 2; Eq 4-6).  Writes (M/bs)*(N/bs) reports and zeroes then fills
+ * *counts (device).  Reference sums are sequential ascending in double (reading R11/R12). */
+aabft_status aabft_check(const aabft_config *cfg, const aabft_encoded *enc,
+                         const aabft_product *prod, aabft_block_report *reports,
+                         aabft_counts *counts, void *ws, size_t ws_bytes, void *stream);
+
+/* Step 4 (reading R15): for every SINGLE block,
+ *   C[i][j] <- Ccol[I][j] - sum_{i' in I, i' != i} C[i'][j]   (double, ascending)
+ * then re-verify row i; status becomes CORRECTED or UNCORRECTABLE and counts are updated. */
+aabft_status aabft_correct(const aabft_config *cfg, const aabft_encoded *enc,
+                           const aabft_product *prod, aabft_block_report *reports,
+                           aabft_counts *counts, void *stream);
+
+/* All four steps on HOST buffers (end-to-end entry point): copies A_host (M x K, dense) and
+ * B_host (K x N, dense) into `arena` (device, >= aabft_host_arena_bytes), runs encode, gemm,
+ * check, correct, and copies C (M x N dense) into C_host and the counts into counts_host.
+ * Host buffers should be pinned for full PCIe bandwidth.  Synchronises `stream`. */
+size_t aabft_host_arena_bytes(const aabft_config *cfg);
+aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_host,
+                                       const void *B_host, void *C_host,
+                                       aabft_counts *counts_host, void *arena,
+                                       size_t arena_bytes, void *stream);
+
+const char *aabft_status_str(aabft_status s);
+/* Thread-local detail for the last non-OK return on this thread. */
+const char *aabft_last_error(void);
+/* Library version string and the number of kernel launches this thread has enqueued
+ * through the library since load (used by bench.py's gpu_launches). */
+const char *aabft_version(void);
+int64_t aabft_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* AABFT_H */

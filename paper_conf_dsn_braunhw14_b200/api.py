@@ -1,0 +1,240 @@
+"""Thin torch-facing binding of the C ABI (include/aabft.h).
+
+Torch provides device memory and the current CUDA stream; every step of the A-ABFT path
+(encode, GEMM, bound, check, correct) runs in the sm_100a kernels of libaabft.so.  This
+module only allocates buffers, builds the ABI structs and forwards pointers.
+
+    plan = ProtectedGemm(M, N, K, dtype=torch.float64, bs=64, p=2)
+    res = plan.run(A, B)             # A, B: CUDA tensors, row-major
+    res.C, res.counts(), res.reports()
+
+``protected_matmul(A, B, ...)`` is the one-shot convenience form (SURVEY §8(b) Python layer).
+"""
+from __future__ import annotations
+
+import ctypes as C
+from dataclasses import dataclass
+
+import numpy as np
+import torch
+
+from . import _abi
+from ._abi import Config, Encoded, Fault, Product, ok, lib
+
+__all__ = ["ProtectedGemm", "protected_matmul", "gemm_plain", "make_faults", "counts_dict"]
+
+
+def _dtype_code(dt: torch.dtype) -> int:
+    if dt == torch.float64:
+        return _abi.F64
+    if dt == torch.float32:
+        return _abi.F32
+    raise TypeError("A-ABFT path supports torch.float64 and torch.float32")
+
+
+def _pad_ld(n: int, dt: torch.dtype) -> int:
+    q = 16 // torch.empty((), dtype=dt).element_size()
+    return (n + q - 1) // q * q
+
+
+def _stream_ptr(stream) -> int:
+    s = torch.cuda.current_stream() if stream is None else stream
+    return s.cuda_stream
+
+
+def _ptr(t) -> int | None:
+    return None if t is None else t.data_ptr()
+
+
+def make_faults(faults, device) -> torch.Tensor | None:
+    """List of dicts (row, col, site, k_step, xor_mask, add) -> device array of aabft_fault."""
+    if not faults:
+        return None
+    arr = np.zeros(len(faults), dtype=_abi.FAULT_DTYPE)
+    for n, f in enumerate(faults):
+        arr[n]["row"] = f["row"]
+        arr[n]["col"] = f["col"]
+        arr[n]["site"] = f.get("site", 0)
+        arr[n]["k_step"] = f.get("k_step", 0)
+        arr[n]["xor_mask"] = np.uint64(f.get("xor_mask", 0))
+        arr[n]["add"] = f.get("add", 0.0)
+    return torch.from_numpy(arr.view(np.uint8).copy()).to(device)
+
+
+def counts_dict(counts: torch.Tensor) -> dict:
+    """Decode an aabft_counts buffer (torch int64[9]) copied to the host."""
+    c = counts.detach().cpu()
+    d = {name: int(c[i]) for i, name in enumerate(_abi.COUNT_NAMES)}
+    d["max_ratio"] = float(c[8:9].view(torch.float64)[0])
+    return d
+
+
+@dataclass
+class Result:
+    C: torch.Tensor
+    Ccol: torch.Tensor
+    Crow: torch.Tensor
+    Acs: torch.Tensor
+    Bcs: torch.Tensor
+    topA_val: torch.Tensor
+    topA_idx: torch.Tensor
+    topB_val: torch.Tensor
+    topB_idx: torch.Tensor
+    report_buf: torch.Tensor
+    counts_buf: torch.Tensor
+    bs: int
+
+    def counts(self) -> dict:
+        return counts_dict(self.counts_buf)
+
+    def reports(self) -> np.ndarray:
+        """Structured numpy array (M/bs, N/bs) with the aabft_block_report fields."""
+        raw = self.report_buf.detach().cpu().numpy()
+        nI = self.C.shape[0] // self.bs
+        return raw.view(_abi.REPORT_DTYPE).reshape(nI, -1)
+
+
+class ProtectedGemm:
+    """Pre-allocated buffers + ABI structs for repeated protected GEMMs of one shape."""
+
+    def __init__(self, M: int, N: int, K: int, *, dtype=torch.float64, bs: int = 64, p: int = 2,
+                 omega: float = 3.0, t: int = 0, fma_model: int = 1, device=None):
+        lib()  # fail loudly before allocating anything
+        self.device = torch.device("cuda" if device is None else device)
+        self.dtype = dtype
+        self.M, self.N, self.K, self.bs, self.p = M, N, K, bs, p
+        self.cfg = Config(_dtype_code(dtype), bs, M, N, K, p, t, omega, fma_model, 0)
+        dev, dt = self.device, dtype
+        nI, nJ = M // bs, N // bs
+        self.ld_acs = _pad_ld(K, dt)
+        self.ld_bcs = _pad_ld(nJ, dt)
+        self.ldc = _pad_ld(N, dt)
+        self.ld_ccol = _pad_ld(N, dt)
+        self.ld_crow = _pad_ld(nJ, dt)
+        self._Acs = torch.empty(nI, self.ld_acs, dtype=dt, device=dev)
+        self._Bcs = torch.empty(K, self.ld_bcs, dtype=dt, device=dev)
+        self._C = torch.empty(M, self.ldc, dtype=dt, device=dev)
+        self._Ccol = torch.empty(nI, self.ld_ccol, dtype=dt, device=dev)
+        self._Crow = torch.empty(M, self.ld_crow, dtype=dt, device=dev)
+        self.topA_val = torch.empty(M + nI, p, dtype=torch.float64, device=dev)
+        self.topA_idx = torch.empty(M + nI, p, dtype=torch.int32, device=dev)
+        self.topB_val = torch.empty(N + nJ, p, dtype=torch.float64, device=dev)
+        self.topB_idx = torch.empty(N + nJ, p, dtype=torch.int32, device=dev)
+        self.reports = torch.empty(nI * nJ * 20, dtype=torch.uint8, device=dev)
+        self.counts = torch.zeros(9, dtype=torch.int64, device=dev)
+        wsb = lib().aabft_workspace_bytes(C.byref(self.cfg))
+        if wsb == 0:
+            ok(1, "aabft_workspace_bytes")
+        self.ws_bytes = int(wsb)
+        self.ws = torch.empty(self.ws_bytes, dtype=torch.uint8, device=dev)
+        self.enc = Encoded(self._Acs.data_ptr(), self.ld_acs, self._Bcs.data_ptr(), self.ld_bcs,
+                           self.topA_val.data_ptr(), self.topA_idx.data_ptr(),
+                           self.topB_val.data_ptr(), self.topB_idx.data_ptr())
+        self.prod = Product(self._C.data_ptr(), self.ldc, self._Ccol.data_ptr(), self.ld_ccol,
+                            self._Crow.data_ptr(), self.ld_crow)
+
+    # views without the pitch padding
+    @property
+    def C(self):
+        return self._C[:, : self.N]
+
+    @property
+    def Ccol(self):
+        return self._Ccol[:, : self.N]
+
+    @property
+    def Crow(self):
+        return self._Crow[:, : self.N // self.bs]
+
+    @property
+    def Acs(self):
+        return self._Acs[:, : self.K]
+
+    @property
+    def Bcs(self):
+        return self._Bcs[:, : self.N // self.bs]
+
+    def _check_operand(self, X, rows, cols, name):
+        if not X.is_cuda or X.dtype != self.dtype or tuple(X.shape) != (rows, cols):
+            raise ValueError(f"{name} must be a CUDA {self.dtype} tensor of shape {(rows, cols)}")
+        if X.stride(1) != 1:
+            raise ValueError(f"{name} must be row-major (stride(1) == 1)")
+
+    # --- the four steps (each one C-ABI call)
+    def encode(self, A, B, stream=None):
+        L = lib()
+        s = _stream_ptr(stream)
+        ok(L.aabft_encode(C.byref(self.cfg), _ptr(A), A.stride(0) if A is not None else 0,
+                          _ptr(B), B.stride(0) if B is not None else 0, C.byref(self.enc),
+                          self.ws.data_ptr(), self.ws_bytes, s), "aabft_encode")
+
+    def gemm(self, A, B, faults: torch.Tensor | None = None, nfaults: int = 0, stream=None):
+        ok(lib().aabft_gemm(C.byref(self.cfg), A.data_ptr(), A.stride(0), B.data_ptr(),
+                            B.stride(0), C.byref(self.enc), C.byref(self.prod), _ptr(faults),
+                            nfaults, self.ws.data_ptr(), self.ws_bytes, _stream_ptr(stream)),
+           "aabft_gemm")
+
+    def check(self, stream=None):
+        ok(lib().aabft_check(C.byref(self.cfg), C.byref(self.enc), C.byref(self.prod),
+                             self.reports.data_ptr(), self.counts.data_ptr(), self.ws.data_ptr(),
+                             self.ws_bytes, _stream_ptr(stream)), "aabft_check")
+
+    def correct(self, stream=None):
+        ok(lib().aabft_correct(C.byref(self.cfg), C.byref(self.enc), C.byref(self.prod),
+                               self.reports.data_ptr(), self.counts.data_ptr(),
+                               _stream_ptr(stream)), "aabft_correct")
+
+    def bound(self, stream=None):
+        nI, nJ = self.M // self.bs, self.N // self.bs
+        eps_col = torch.empty(nI, self.N, dtype=torch.float64, device=self.device)
+        sig_col = torch.empty_like(eps_col)
+        eps_row = torch.empty(self.M, nJ, dtype=torch.float64, device=self.device)
+        sig_row = torch.empty_like(eps_row)
+        ok(lib().aabft_bound(C.byref(self.cfg), C.byref(self.enc), eps_col.data_ptr(),
+                             sig_col.data_ptr(), eps_row.data_ptr(), sig_row.data_ptr(),
+                             _stream_ptr(stream)), "aabft_bound")
+        return dict(eps_col=eps_col, sig_col=sig_col, eps_row=eps_row, sig_row=sig_row)
+
+    def run(self, A, B, *, faults=None, correct: bool = True, stream=None) -> Result:
+        """encode -> gemm -> check -> correct, all enqueued on one stream."""
+        self._check_operand(A, self.M, self.K, "A")
+        self._check_operand(B, self.K, self.N, "B")
+        fbuf = faults if isinstance(faults, torch.Tensor) else make_faults(faults, self.device)
+        nf = 0 if fbuf is None else fbuf.numel() // 48
+        self.encode(A, B, stream)
+        self.gemm(A, B, fbuf, nf, stream)
+        self.check(stream)
+        if correct:
+            self.correct(stream)
+        return self.result()
+
+    def result(self) -> Result:
+        return Result(self.C, self.Ccol, self.Crow, self.Acs, self.Bcs, self.topA_val,
+                      self.topA_idx, self.topB_val, self.topB_idx, self.reports, self.counts,
+                      self.bs)
+
+
+def protected_matmul(A, B, *, bs: int = 64, p: int = 2, omega: float = 3.0, t: int = 0,
+                     fma_model: int = 1, correct: bool = True, faults=None) -> Result:
+    """One-shot A-ABFT protected C = A @ B on the current CUDA stream."""
+    M, K = A.shape
+    N = B.shape[1]
+    plan = ProtectedGemm(M, N, K, dtype=A.dtype, bs=bs, p=p, omega=omega, t=t,
+                         fma_model=fma_model, device=A.device)
+    return plan.run(A, B, faults=faults, correct=correct)
+
+
+def gemm_plain(A, B, out=None, stream=None):
+    """Unprotected C = A @ B with the same kernel family (overhead denominator)."""
+    M, K = A.shape
+    N = B.shape[1]
+    dt = A.dtype
+    if out is None:
+        out = torch.empty(M, _pad_ld(N, dt), dtype=dt, device=A.device)
+    cfg = Config(_dtype_code(dt), 8, M, N, K, 1, 0, 3.0, 1, 0)  # bs=8: validation only
+    if M % 8 or N % 8:
+        raise ValueError("gemm_plain: M and N must be multiples of 8")
+    ok(lib().aabft_gemm_plain(C.byref(cfg), A.data_ptr(), A.stride(0), B.data_ptr(), B.stride(0),
+                              out.data_ptr(), out.stride(0), _stream_ptr(stream)),
+       "aabft_gemm_plain")
+    return out[:, :N]

@@ -1,0 +1,345 @@
+// api.cu -- the C ABI of include/aabft.h: validation, workspace sizing, dispatch, errors.
+// No C++ exception crosses the ABI; every entry point is stream-ordered and never allocates.
+#include <atomic>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+
+#include "common.cuh"
+
+namespace aabft {
+
+size_t encode_ws_bytes(const aabft_config *cfg);
+
+namespace {
+thread_local char g_err[512] = "";
+std::atomic<int64_t> g_launches{0};
+int g_dev_ok[64] = {0};  // 0 unknown, 1 ok, 2 unsupported
+
+inline size_t r256(size_t b) { return (b + 255) / 256 * 256; }
+
+bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
+}  // namespace
+
+void set_error(const char *fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_err, sizeof g_err, fmt, ap);
+  va_end(ap);
+}
+
+int64_t next_launch(int64_t n) { return g_launches.fetch_add(n) + n; }
+
+aabft_status check_launch(const char *what) {
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) {
+    set_error("%s: %s", what, cudaGetErrorString(e));
+    return AABFT_ECUDA;
+  }
+  return AABFT_OK;
+}
+
+int eff_t(const aabft_config *cfg) {
+  if (cfg->t > 0) return cfg->t;
+  return cfg->dtype == AABFT_F64 ? 52 : 23;
+}
+
+size_t elem_size(const aabft_config *cfg) { return cfg->dtype == AABFT_F64 ? 8 : 4; }
+
+double sigma_coeff(int64_t K, int fma_model) {
+  const double dn = (double)K;
+  double F;
+  if (fma_model) F = ((dn * (dn + 1.0)) * (2.0 * dn + 1.0)) / 48.0;
+  else F = ((dn * (dn + 1.0)) * (dn + 0.5) + 2.0 * dn) / 24.0;
+  return std::sqrt(F);
+}
+
+BoundParams make_bound_params(const aabft_config *cfg) {
+  BoundParams b;
+  const int t = eff_t(cfg);
+  b.s = sigma_coeff(cfg->K, cfg->fma_model);
+  b.two_mt = std::ldexp(1.0, -t);
+  b.two_m2t = std::ldexp(1.0, -2 * t);
+  b.omega = cfg->omega;
+  b.ev_coeff = (double)cfg->K / 3.0;
+  b.fma_model = cfg->fma_model;
+  b.p = cfg->p;
+  return b;
+}
+
+aabft_status validate(const aabft_config *c) {
+  if (!c) { set_error("config is NULL"); return AABFT_EINVAL; }
+  if (c->dtype != AABFT_F64 && c->dtype != AABFT_F32) { set_error("dtype %d", c->dtype); return AABFT_EINVAL; }
+  if (c->M < 1 || c->N < 1 || c->K < 1) { set_error("M, N, K must be >= 1"); return AABFT_EINVAL; }
+  if (c->K >= (int64_t)1 << 31) { set_error("K must be < 2^31"); return AABFT_EINVAL; }
+  if (c->bs < 8 || c->bs > 256 || (c->bs & (c->bs - 1))) { set_error("bs=%d must be a power of 2 in [8,256]", c->bs); return AABFT_EINVAL; }
+  if (c->M % c->bs || c->N % c->bs) { set_error("M and N must be multiples of bs (zero-pad, P:L353)"); return AABFT_EINVAL; }
+  if (c->p < 1 || c->p > 8 || c->p > c->K) { set_error("p=%d must be in [1, min(8, K)]", c->p); return AABFT_EINVAL; }
+  if (!(c->omega > 0.0) || !std::isfinite(c->omega)) { set_error("omega must be positive and finite"); return AABFT_EINVAL; }
+  if (c->t < 0 || c->t > 200) { set_error("t=%d out of range", c->t); return AABFT_EINVAL; }
+  if (c->fma_model != 0 && c->fma_model != 1) { set_error("fma_model must be 0 or 1"); return AABFT_EINVAL; }
+  if ((c->M / c->bs) * (c->N / c->bs) >= ((int64_t)1 << 31)) { set_error("too many blocks"); return AABFT_EINVAL; }
+  return AABFT_OK;
+}
+
+static aabft_status device_ok() {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return check_launch("cudaGetDevice");
+  if (dev < 0 || dev >= 64) return AABFT_EUNSUPPORTED;
+  if (g_dev_ok[dev] == 0) {
+    int major = 0, minor = 0;
+    cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev);
+    cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev);
+    g_dev_ok[dev] = (major == 10 && minor == 0) ? 1 : 2;
+    if (g_dev_ok[dev] == 2) set_error("device %d is sm_%d%d; this library is built for sm_100a", dev, major, minor);
+  }
+  if (g_dev_ok[dev] != 1) {
+    set_error("device is not sm_100 (B200); library built for sm_100a only");
+    return AABFT_EUNSUPPORTED;
+  }
+  return AABFT_OK;
+}
+
+// rows of a row-major operand fed to TMA / vector loads: base 16-B aligned, pitch 16-B multiple
+static bool pitch_ok(const aabft_config *c, const void *p, int64_t ld) {
+  return aligned16(p) && ((size_t)ld * elem_size(c)) % 16 == 0;
+}
+
+}  // namespace aabft
+
+using namespace aabft;
+
+#define AABFT_GUARD_BEGIN try {
+#define AABFT_GUARD_END                                     \
+  }                                                         \
+  catch (...) {                                             \
+    set_error("internal error (exception caught at ABI)"); \
+    return AABFT_EINTERNAL;                                 \
+  }
+
+extern "C" {
+
+size_t aabft_workspace_bytes(const aabft_config *cfg) {
+  if (validate(cfg) != AABFT_OK) return 0;
+  return r256(encode_ws_bytes(cfg)) + 256;
+}
+
+aabft_status aabft_encode(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
+                          int64_t ldb, const aabft_encoded *out, void *ws, size_t ws_bytes,
+                          void *stream) {
+  AABFT_GUARD_BEGIN
+  aabft_status s = validate(cfg);
+  if (s != AABFT_OK) return s;
+  if (!out) { set_error("out is NULL"); return AABFT_EINVAL; }
+  if (!A && !B) { set_error("A and B are both NULL"); return AABFT_EINVAL; }
+  if (A && (lda < cfg->K || !out->Acs || out->ld_acs < cfg->K || !out->topA_val || !out->topA_idx)) {
+    set_error("encode A: need lda >= K, Acs (ld_acs >= K), topA_val, topA_idx");
+    return AABFT_EINVAL;
+  }
+  if (B && (ldb < cfg->N || !out->Bcs || out->ld_bcs < cfg->N / cfg->bs || !out->topB_val || !out->topB_idx)) {
+    set_error("encode B: need ldb >= N, Bcs (ld_bcs >= N/bs), topB_val, topB_idx");
+    return AABFT_EINVAL;
+  }
+  if (!ws || ws_bytes < aabft_workspace_bytes(cfg)) {
+    set_error("workspace too small: need %zu bytes", aabft_workspace_bytes(cfg));
+    return AABFT_EWORKSPACE;
+  }
+  if ((s = device_ok()) != AABFT_OK) return s;
+  return launch_encode(cfg, A, lda, B, ldb, out, ws, (cudaStream_t)stream);
+  AABFT_GUARD_END
+}
+
+aabft_status aabft_bound(const aabft_config *cfg, const aabft_encoded *enc, double *eps_col,
+                         double *sig_col, double *eps_row, double *sig_row, void *stream) {
+  AABFT_GUARD_BEGIN
+  aabft_status s = validate(cfg);
+  if (s != AABFT_OK) return s;
+  if (!enc || !enc->topA_val || !enc->topA_idx || !enc->topB_val || !enc->topB_idx) {
+    set_error("bound: top-p tables required");
+    return AABFT_EINVAL;
+  }
+  if ((s = device_ok()) != AABFT_OK) return s;
+  return launch_bound(cfg, enc, eps_col, sig_col, eps_row, sig_row, (cudaStream_t)stream);
+  AABFT_GUARD_END
+}
+
+static aabft_status gemm_common(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
+                                int64_t ldb, const aabft_encoded *enc, const aabft_product *out,
+                                const aabft_fault *faults, int32_t nfaults, bool plain,
+                                void *stream) {
+  aabft_status s = validate(cfg);
+  if (s != AABFT_OK) return s;
+  if (!A || !B || !out || !out->C) { set_error("gemm: A, B, C required"); return AABFT_EINVAL; }
+  if (lda < cfg->K || ldb < cfg->N || out->ldc < cfg->N) { set_error("gemm: lda >= K, ldb >= N, ldc >= N required"); return AABFT_EINVAL; }
+  if (!pitch_ok(cfg, A, lda) || !pitch_ok(cfg, B, ldb) || !aligned16(out->C)) {
+    set_error("gemm: A/B/C must be 16-byte aligned with row pitches that are multiples of 16 bytes");
+    return AABFT_EINVAL;
+  }
+  if (!plain) {
+    if (!enc || !enc->Acs || !enc->Bcs || !out->Ccol || !out->Crow) { set_error("gemm: Acs, Bcs, Ccol, Crow required"); return AABFT_EINVAL; }
+    if (enc->ld_acs < cfg->K || enc->ld_bcs < cfg->N / cfg->bs || out->ld_ccol < cfg->N || out->ld_crow < cfg->N / cfg->bs) {
+      set_error("gemm: checksum leading dimensions too small");
+      return AABFT_EINVAL;
+    }
+    if (!pitch_ok(cfg, enc->Acs, enc->ld_acs) || !pitch_ok(cfg, enc->Bcs, enc->ld_bcs)) {
+      set_error("gemm: Acs/Bcs must be 16-byte aligned with 16-byte-multiple row pitches (pad ld_bcs)");
+      return AABFT_EINVAL;
+    }
+    if (nfaults < 0 || (nfaults > 0 && !faults)) { set_error("gemm: bad fault list"); return AABFT_EINVAL; }
+  }
+  if ((s = device_ok()) != AABFT_OK) return s;
+  if (cfg->dtype == AABFT_F64)
+    return launch_gemm_f64(cfg, A, lda, B, ldb, enc, out, plain ? nullptr : faults, plain ? 0 : nfaults, plain, (cudaStream_t)stream);
+  return launch_gemm_f32(cfg, A, lda, B, ldb, enc, out, plain ? nullptr : faults, plain ? 0 : nfaults, plain, (cudaStream_t)stream);
+}
+
+aabft_status aabft_gemm(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
+                        int64_t ldb, const aabft_encoded *enc, const aabft_product *out,
+                        const aabft_fault *faults, int32_t nfaults, void *ws, size_t ws_bytes,
+                        void *stream) {
+  AABFT_GUARD_BEGIN
+  (void)ws;
+  (void)ws_bytes;
+  return gemm_common(cfg, A, lda, B, ldb, enc, out, faults, nfaults, false, stream);
+  AABFT_GUARD_END
+}
+
+aabft_status aabft_gemm_plain(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
+                              int64_t ldb, void *C, int64_t ldc, void *stream) {
+  AABFT_GUARD_BEGIN
+  aabft_product out{};
+  out.C = C;
+  out.ldc = ldc;
+  return gemm_common(cfg, A, lda, B, ldb, nullptr, &out, nullptr, 0, true, stream);
+  AABFT_GUARD_END
+}
+
+static aabft_status check_common(const aabft_config *cfg, const aabft_encoded *enc,
+                                 const aabft_product *prod, aabft_block_report *rep,
+                                 aabft_counts *cnt) {
+  aabft_status s = validate(cfg);
+  if (s != AABFT_OK) return s;
+  if (!enc || !enc->topA_val || !enc->topA_idx || !enc->topB_val || !enc->topB_idx) { set_error("check: top-p tables required"); return AABFT_EINVAL; }
+  if (!prod || !prod->C || !prod->Ccol || !prod->Crow || !rep || !cnt) { set_error("check: C, Ccol, Crow, reports, counts required"); return AABFT_EINVAL; }
+  if (prod->ldc < cfg->N || prod->ld_ccol < cfg->N || prod->ld_crow < cfg->N / cfg->bs) { set_error("check: leading dimensions too small"); return AABFT_EINVAL; }
+  return device_ok();
+}
+
+aabft_status aabft_check(const aabft_config *cfg, const aabft_encoded *enc,
+                         const aabft_product *prod, aabft_block_report *reports,
+                         aabft_counts *counts, void *ws, size_t ws_bytes, void *stream) {
+  AABFT_GUARD_BEGIN
+  (void)ws;
+  (void)ws_bytes;
+  aabft_status s = check_common(cfg, enc, prod, reports, counts);
+  if (s != AABFT_OK) return s;
+  return launch_check(cfg, enc, prod, reports, counts, (cudaStream_t)stream);
+  AABFT_GUARD_END
+}
+
+aabft_status aabft_correct(const aabft_config *cfg, const aabft_encoded *enc,
+                           const aabft_product *prod, aabft_block_report *reports,
+                           aabft_counts *counts, void *stream) {
+  AABFT_GUARD_BEGIN
+  aabft_status s = check_common(cfg, enc, prod, reports, counts);
+  if (s != AABFT_OK) return s;
+  return launch_correct(cfg, enc, prod, reports, counts, (cudaStream_t)stream);
+  AABFT_GUARD_END
+}
+
+// ------------------------------------------------------------------ host end-to-end entry point
+namespace {
+struct Arena {
+  int64_t lda, ldb, ldc, ld_acs, ld_bcs, ld_ccol, ld_crow;
+  size_t oA, oB, oC, oAcs, oBcs, oCcol, oCrow, oTav, oTai, oTbv, oTbi, oRep, oCnt, oWs, total;
+};
+Arena plan_arena(const aabft_config *c) {
+  Arena a;
+  const size_t es = elem_size(c);
+  const int64_t q = 16 / (int64_t)es;  // elements per 16 bytes
+  auto rnd = [q](int64_t n) { return (n + q - 1) / q * q; };
+  a.lda = rnd(c->K); a.ldb = rnd(c->N); a.ldc = rnd(c->N);
+  a.ld_acs = rnd(c->K); a.ld_bcs = rnd(c->N / c->bs);
+  a.ld_ccol = rnd(c->N); a.ld_crow = rnd(c->N / c->bs);
+  size_t o = 0;
+  auto take = [&o](size_t bytes) { size_t r = o; o += r256(bytes); return r; };
+  a.oA = take(c->M * a.lda * es);
+  a.oB = take(c->K * a.ldb * es);
+  a.oC = take(c->M * a.ldc * es);
+  a.oAcs = take((c->M / c->bs) * a.ld_acs * es);
+  a.oBcs = take(c->K * a.ld_bcs * es);
+  a.oCcol = take((c->M / c->bs) * a.ld_ccol * es);
+  a.oCrow = take(c->M * a.ld_crow * es);
+  a.oTav = take((c->M + c->M / c->bs) * c->p * 8);
+  a.oTai = take((c->M + c->M / c->bs) * c->p * 4);
+  a.oTbv = take((c->N + c->N / c->bs) * c->p * 8);
+  a.oTbi = take((c->N + c->N / c->bs) * c->p * 4);
+  a.oRep = take((c->M / c->bs) * (c->N / c->bs) * sizeof(aabft_block_report));
+  a.oCnt = take(sizeof(aabft_counts));
+  a.oWs = take(aabft_workspace_bytes(c));
+  a.total = o;
+  return a;
+}
+}  // namespace
+
+size_t aabft_host_arena_bytes(const aabft_config *cfg) {
+  if (validate(cfg) != AABFT_OK) return 0;
+  return plan_arena(cfg).total;
+}
+
+aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_host,
+                                       const void *B_host, void *C_host,
+                                       aabft_counts *counts_host, void *arena,
+                                       size_t arena_bytes, void *stream) {
+  AABFT_GUARD_BEGIN
+  aabft_status s = validate(cfg);
+  if (s != AABFT_OK) return s;
+  if (!A_host || !B_host || !C_host) { set_error("host buffers required"); return AABFT_EINVAL; }
+  const Arena a = plan_arena(cfg);
+  if (!arena || arena_bytes < a.total) { set_error("arena too small: need %zu bytes", a.total); return AABFT_EWORKSPACE; }
+  if (!aligned16(arena)) { set_error("arena must be 16-byte aligned"); return AABFT_EINVAL; }
+  cudaStream_t st = (cudaStream_t)stream;
+  char *base = static_cast<char *>(arena);
+  const size_t es = elem_size(cfg);
+  if (cudaMemcpy2DAsync(base + a.oA, a.lda * es, A_host, cfg->K * es, cfg->K * es, cfg->M, cudaMemcpyHostToDevice, st) != cudaSuccess ||
+      cudaMemcpy2DAsync(base + a.oB, a.ldb * es, B_host, cfg->N * es, cfg->N * es, cfg->K, cudaMemcpyHostToDevice, st) != cudaSuccess)
+    return check_launch("host->device copy");
+  aabft_encoded enc{base + a.oAcs, a.ld_acs, base + a.oBcs, a.ld_bcs,
+                    reinterpret_cast<double *>(base + a.oTav), reinterpret_cast<int32_t *>(base + a.oTai),
+                    reinterpret_cast<double *>(base + a.oTbv), reinterpret_cast<int32_t *>(base + a.oTbi)};
+  aabft_product prod{base + a.oC, a.ldc, base + a.oCcol, a.ld_ccol, base + a.oCrow, a.ld_crow};
+  auto *rep = reinterpret_cast<aabft_block_report *>(base + a.oRep);
+  auto *cnt = reinterpret_cast<aabft_counts *>(base + a.oCnt);
+  const size_t wsb = aabft_workspace_bytes(cfg);
+  if ((s = aabft_encode(cfg, base + a.oA, a.lda, base + a.oB, a.ldb, &enc, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
+  if ((s = aabft_gemm(cfg, base + a.oA, a.lda, base + a.oB, a.ldb, &enc, &prod, nullptr, 0, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
+  if ((s = aabft_check(cfg, &enc, &prod, rep, cnt, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
+  if ((s = aabft_correct(cfg, &enc, &prod, rep, cnt, stream)) != AABFT_OK) return s;
+  if (cudaMemcpy2DAsync(C_host, cfg->N * es, base + a.oC, a.ldc * es, cfg->N * es, cfg->M, cudaMemcpyDeviceToHost, st) != cudaSuccess)
+    return check_launch("device->host copy");
+  if (counts_host && cudaMemcpyAsync(counts_host, cnt, sizeof(aabft_counts), cudaMemcpyDeviceToHost, st) != cudaSuccess)
+    return check_launch("counts copy");
+  if (cudaStreamSynchronize(st) != cudaSuccess) return check_launch("stream sync");
+  return AABFT_OK;
+  AABFT_GUARD_END
+}
+
+const char *aabft_status_str(aabft_status s) {
+  switch (s) {
+    case AABFT_OK: return "AABFT_OK";
+    case AABFT_EINVAL: return "AABFT_EINVAL: invalid argument";
+    case AABFT_EUNSUPPORTED: return "AABFT_EUNSUPPORTED: device is not sm_100";
+    case AABFT_ECUDA: return "AABFT_ECUDA: CUDA error";
+    case AABFT_EWORKSPACE: return "AABFT_EWORKSPACE: workspace missing or too small";
+    case AABFT_EINTERNAL: return "AABFT_EINTERNAL: internal error";
+  }
+  return "unknown aabft_status";
+}
+
+const char *aabft_last_error(void) { return g_err; }
+const char *aabft_version(void) { return "aabft-b200 0.1 (sm_100a; DMMA f64 / FFMA f32)"; }
+int64_t aabft_launch_count(void) { return g_launches.load(); }
+
+}  // extern "C"

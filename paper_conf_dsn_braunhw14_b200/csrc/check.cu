@@ -1,0 +1,354 @@
+// check.cu -- steps 4a-4c and the correction of Alg 2 on sm_100a.
+//
+// Bound (§IV-E): per carried checksum element, y from the top-p lists of the two
+// vectors of its inner product (three cases, reading R3), sigma = sqrt(F(K)) y 2^-t
+// (Eq 28 P:L219 / P:L287), eps = omega sigma (Eq 7) (+ |EV_Prod| Eq 43 when
+// fma_model = 0).  Evaluated in double with explicit round-to-nearest intrinsics so no FMA
+// contraction can change a bit (bit-identical to the definition).
+//
+// Check (Eq 4-6): one CTA per BS x BS sub-matrix of C (as Alg 2).  The block is
+// streamed in 32-row strips through padded shared memory: a thread per column keeps the
+// reference column sum in a register (ascending i) and a thread per row sums its strip row
+// (ascending j); both in double (readings R11/R12).  Classification (R9/R10):
+// ROUNDING |d| <= sigma, TOLERABLE <= eps, CRITICAL otherwise (NaN/Inf included).
+#include <algorithm>
+#include <cfloat>
+#include <math_constants.h>
+
+#include "common.cuh"
+
+namespace aabft {
+namespace {
+
+constexpr int kCheckThreads = 256;
+constexpr int kCheckStrip = 32;
+
+template <int P>
+__device__ __forceinline__ double y_bound(const double *__restrict__ va, const int *__restrict__ ia,
+                                          const double *__restrict__ vb,
+                                          const int *__restrict__ ib) {
+  double a[P], b[P];
+  int ai[P], bi[P];
+#pragma unroll
+  for (int r = 0; r < P; ++r) { a[r] = va[r]; b[r] = vb[r]; ai[r] = ia[r]; bi[r] = ib[r]; }
+  double case1 = 0.0;
+#pragma unroll
+  for (int r = 0; r < P; ++r)
+#pragma unroll
+    for (int s = 0; s < P; ++s)
+      if (ai[r] == bi[s]) case1 = fmax(case1, __dmul_rn(a[r], b[s]));
+  double amax = a[0], amin = a[0], bmax = b[0], bmin = b[0];
+#pragma unroll
+  for (int r = 1; r < P; ++r) {
+    amax = fmax(amax, a[r]); amin = fmin(amin, a[r]);
+    bmax = fmax(bmax, b[r]); bmin = fmin(bmin, b[r]);
+  }
+  return fmax(case1, fmax(__dmul_rn(amax, bmin), __dmul_rn(bmax, amin)));
+}
+
+struct Bound {
+  double sig, eps;
+};
+__device__ __forceinline__ Bound bound_of(const BoundParams &bp, double y) {
+  Bound b;
+  b.sig = __dmul_rn(bp.s, __dmul_rn(y, bp.two_mt));
+  b.eps = __dmul_rn(bp.omega, b.sig);
+  if (!bp.fma_model) b.eps = __dadd_rn(b.eps, __dmul_rn(bp.ev_coeff, __dmul_rn(y, bp.two_m2t)));
+  return b;
+}
+
+__device__ __forceinline__ int classify(double d, const Bound &b) {
+  const double a = fabs(d);
+  if (a <= b.sig) return 0;
+  if (a <= b.eps) return 1;
+  return 2;  // !(|d| <= eps): NaN and Inf are critical (reading R9)
+}
+__device__ __forceinline__ double ratio_of(double d, double eps) {
+  const double a = fabs(d);
+  if (a != a) return CUDART_INF;
+  if (eps > 0.0) return a / eps;
+  return a == 0.0 ? 0.0 : CUDART_INF;
+}
+
+// atomic max on non-negative doubles (bit pattern order == value order)
+__device__ __forceinline__ void atomic_max_nonneg(double *addr, double v) {
+  atomicMax(reinterpret_cast<unsigned long long *>(addr),
+            (unsigned long long)__double_as_longlong(v));
+}
+
+// --------------------------------------------------------------------------- bound only
+template <int P>
+__global__ void bound_kernel(int64_t M, int64_t N, int bs, BoundParams bp,
+                             const double *__restrict__ tav, const int *__restrict__ tai,
+                             const double *__restrict__ tbv, const int *__restrict__ tbi,
+                             double *eps_col, double *sig_col, double *eps_row,
+                             double *sig_row) {
+  const int64_t ncol = (M / bs) * N, nrow = M * (N / bs);
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < ncol + nrow;
+       e += (int64_t)gridDim.x * blockDim.x) {
+    if (e < ncol) {
+      const int64_t I = e / N, j = e % N;
+      const double y = y_bound<P>(tav + (M + I) * P, tai + (M + I) * P, tbv + j * P, tbi + j * P);
+      const Bound b = bound_of(bp, y);
+      if (eps_col) eps_col[e] = b.eps;
+      if (sig_col) sig_col[e] = b.sig;
+    } else {
+      const int64_t f = e - ncol, nJ = N / bs, i = f / nJ, J = f % nJ;
+      const double y = y_bound<P>(tav + i * P, tai + i * P, tbv + (N + J) * P, tbi + (N + J) * P);
+      const Bound b = bound_of(bp, y);
+      if (eps_row) eps_row[f] = b.eps;
+      if (sig_row) sig_row[f] = b.sig;
+    }
+  }
+}
+
+// --------------------------------------------------------------------------- check
+struct CheckArgs {
+  int64_t M, N;
+  int bs;
+  const void *C;
+  int64_t ldc;
+  const void *Ccol;
+  int64_t ld_ccol;
+  const void *Crow;
+  int64_t ld_crow;
+  const double *tav;
+  const int *tai;
+  const double *tbv;
+  const int *tbi;
+  aabft_block_report *rep;
+  aabft_counts *cnt;
+};
+
+template <typename T, int P>
+__global__ void __launch_bounds__(kCheckThreads) check_kernel(CheckArgs a, BoundParams bp) {
+  extern __shared__ double tile[];  // kCheckStrip x (bs + 1)
+  __shared__ int s_cls[3], s_nr, s_nc, s_row, s_col;
+  __shared__ double s_ratio[kCheckThreads / 32];
+  const int bs = a.bs, tid = threadIdx.x, lane = tid & 31;
+  const int64_t nJ = a.N / bs;
+  const int64_t I = blockIdx.x / nJ, J = blockIdx.x % nJ;
+  const T *C = static_cast<const T *>(a.C);
+  if (tid < 3) s_cls[tid] = 0;
+  if (tid == 0) { s_nr = 0; s_nc = 0; s_row = -1; s_col = -1; }
+  const int stride = bs + 1;
+  const int rs = min(bs, kCheckStrip);
+  double colsum = 0.0;
+  int cls_local[3] = {0, 0, 0};
+  double rmax = 0.0;
+  const int row_worker = tid - (kCheckThreads - kCheckStrip);  // last warp sums rows
+  for (int r0 = 0; r0 < bs; r0 += rs) {
+    // coalesced strip load: rs rows x bs columns
+    for (int e = tid; e < rs * bs; e += kCheckThreads) {
+      const int rr = e / bs, cc = e % bs;
+      tile[rr * stride + cc] = (double)C[(I * bs + r0 + rr) * a.ldc + J * bs + cc];
+    }
+    __syncthreads();
+    if (tid < bs) {
+      for (int rr = 0; rr < rs; ++rr) colsum = colsum + tile[rr * stride + tid];  // Eq 4, asc i
+    }
+    if (row_worker >= 0 && row_worker < rs) {
+      const int64_t i = I * bs + r0 + row_worker;
+      double ref = 0.0;
+      for (int cc = 0; cc < bs; ++cc) ref = ref + tile[row_worker * stride + cc];  // asc j
+      const double carried = (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
+      const double d = ref - carried;
+      const double y = y_bound<P>(a.tav + i * P, a.tai + i * P, a.tbv + (a.N + J) * P,
+                                  a.tbi + (a.N + J) * P);
+      const Bound b = bound_of(bp, y);
+      const int cl = classify(d, b);
+      cls_local[cl] += 1;
+      if (cl == 2) { atomicAdd(&s_nr, 1); s_row = (int)i; }
+      rmax = fmax(rmax, ratio_of(d, b.eps));
+    }
+    __syncthreads();
+  }
+  if (tid < bs) {
+    const int64_t j = J * bs + tid;
+    const double carried = (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
+    const double d = colsum - carried;
+    const double y = y_bound<P>(a.tav + (a.M + I) * P, a.tai + (a.M + I) * P, a.tbv + j * P,
+                                a.tbi + j * P);
+    const Bound b = bound_of(bp, y);
+    const int cl = classify(d, b);
+    cls_local[cl] += 1;
+    if (cl == 2) { atomicAdd(&s_nc, 1); s_col = (int)j; }
+    rmax = fmax(rmax, ratio_of(d, b.eps));
+  }
+  // block reductions
+#pragma unroll
+  for (int c = 0; c < 3; ++c) {
+    int v = cls_local[c];
+#pragma unroll
+    for (int m = 16; m >= 1; m >>= 1) v += __shfl_xor_sync(0xffffffffu, v, m);
+    if (lane == 0 && v) atomicAdd(&s_cls[c], v);
+  }
+#pragma unroll
+  for (int m = 16; m >= 1; m >>= 1) rmax = fmax(rmax, __shfl_xor_sync(0xffffffffu, rmax, m));
+  if (lane == 0) s_ratio[tid >> 5] = rmax;
+  __syncthreads();
+  if (tid == 0) {
+    double br = 0.0;
+    for (int w = 0; w < kCheckThreads / 32; ++w) br = fmax(br, s_ratio[w]);
+    const int nr = s_nr, nc = s_nc;
+    uint8_t status;
+    if (nr == 0 && nc == 0) status = AABFT_BLK_CLEAN;
+    else if (nr == 1 && nc == 1) status = AABFT_BLK_SINGLE;
+    else if (nr == 0 || nc == 0) status = AABFT_BLK_CHECKSUM_ONLY;
+    else status = AABFT_BLK_UNCORRECTABLE;
+    aabft_block_report r;
+    r.status = status;
+    r.worst_class = (uint8_t)(s_cls[2] ? 2 : (s_cls[1] ? 1 : 0));
+    r.n_bad_rows = (uint16_t)min(nr, 65535);
+    r.n_bad_cols = (uint16_t)min(nc, 65535);
+    r.reserved = 0;
+    r.row = status == AABFT_BLK_SINGLE ? s_row : -1;
+    r.col = status == AABFT_BLK_SINGLE ? s_col : -1;
+    r.max_ratio = (float)br;
+    a.rep[blockIdx.x] = r;
+    unsigned long long *n = reinterpret_cast<unsigned long long *>(a.cnt->n);
+    atomicAdd(&n[0], 1ull);
+    if (status == AABFT_BLK_CLEAN) atomicAdd(&n[1], 1ull);
+    if (status == AABFT_BLK_CHECKSUM_ONLY) atomicAdd(&n[3], 1ull);
+    if (status == AABFT_BLK_UNCORRECTABLE) atomicAdd(&n[4], 1ull);
+    for (int c = 0; c < 3; ++c)
+      if (s_cls[c]) atomicAdd(&n[5 + c], (unsigned long long)s_cls[c]);
+    if (br > 0.0) atomic_max_nonneg(&a.cnt->max_ratio, br);
+  }
+}
+
+// --------------------------------------------------------------------------- correct
+template <typename T, int P>
+__global__ void correct_kernel(CheckArgs a, BoundParams bp, T *C) {
+  const int bs = a.bs;
+  const int64_t nJ = a.N / bs, nb = (a.M / bs) * nJ;
+  for (int64_t blk = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; blk < nb;
+       blk += (int64_t)gridDim.x * blockDim.x) {
+    aabft_block_report *r = a.rep + blk;
+    if (r->status != AABFT_BLK_SINGLE) continue;
+    const int64_t I = blk / nJ, J = blk % nJ, i = r->row, j = r->col;
+    // c_ij <- Ccol[I][j] - sum_{i' != i} c_i'j  (reading R15; double, ascending i')
+    double v = (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
+    for (int64_t ii = I * bs; ii < I * bs + bs; ++ii)
+      if (ii != i) v = v - (double)C[ii * a.ldc + j];
+    C[i * a.ldc + j] = (T)v;
+    // re-verify row i
+    double ref = 0.0;
+    for (int64_t jj = J * bs; jj < J * bs + bs; ++jj) ref = ref + (double)C[i * a.ldc + jj];
+    const double d = ref - (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
+    const double y = y_bound<P>(a.tav + i * P, a.tai + i * P, a.tbv + (a.N + J) * P,
+                                a.tbi + (a.N + J) * P);
+    const Bound b = bound_of(bp, y);
+    unsigned long long *n = reinterpret_cast<unsigned long long *>(a.cnt->n);
+    if (fabs(d) <= b.eps) {
+      r->status = AABFT_BLK_CORRECTED;
+      atomicAdd(&n[2], 1ull);
+    } else {
+      r->status = AABFT_BLK_UNCORRECTABLE;
+      atomicAdd(&n[4], 1ull);
+    }
+  }
+}
+
+CheckArgs make_args(const aabft_config *cfg, const aabft_encoded *enc, const aabft_product *prod,
+                    aabft_block_report *rep, aabft_counts *cnt) {
+  CheckArgs a;
+  a.M = cfg->M; a.N = cfg->N; a.bs = cfg->bs;
+  a.C = prod->C; a.ldc = prod->ldc;
+  a.Ccol = prod->Ccol; a.ld_ccol = prod->ld_ccol;
+  a.Crow = prod->Crow; a.ld_crow = prod->ld_crow;
+  a.tav = enc->topA_val; a.tai = enc->topA_idx;
+  a.tbv = enc->topB_val; a.tbi = enc->topB_idx;
+  a.rep = rep; a.cnt = cnt;
+  return a;
+}
+
+template <typename T, int P>
+aabft_status run_check(const aabft_config *cfg, const CheckArgs &a, BoundParams bp,
+                       cudaStream_t st) {
+  const int64_t nb = (cfg->M / cfg->bs) * (cfg->N / cfg->bs);
+  const size_t smem = (size_t)kCheckStrip * (cfg->bs + 1) * sizeof(double);
+  auto kern = check_kernel<T, P>;
+  if (smem > 48 * 1024) {
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  }
+  if (nb > 0) {
+    kern<<<(unsigned)nb, kCheckThreads, smem, st>>>(a, bp);
+    next_launch();
+  }
+  return check_launch("aabft_check");
+}
+
+template <typename T, int P>
+aabft_status run_correct(const aabft_config *cfg, const CheckArgs &a, BoundParams bp,
+                         cudaStream_t st) {
+  const int64_t nb = (cfg->M / cfg->bs) * (cfg->N / cfg->bs);
+  const unsigned grid = (unsigned)std::min<int64_t>((nb + 255) / 256, 4096);
+  if (nb > 0) {
+    correct_kernel<T, P><<<grid, 256, 0, st>>>(a, bp, static_cast<T *>(const_cast<void *>(a.C)));
+    next_launch();
+  }
+  return check_launch("aabft_correct");
+}
+
+#define AABFT_P_SWITCH(p, ...)          \
+  switch (p) {                           \
+    case 1: { constexpr int PP = 1; __VA_ARGS__; } \
+    case 2: { constexpr int PP = 2; __VA_ARGS__; } \
+    case 3: { constexpr int PP = 3; __VA_ARGS__; } \
+    case 4: { constexpr int PP = 4; __VA_ARGS__; } \
+    case 5: { constexpr int PP = 5; __VA_ARGS__; } \
+    case 6: { constexpr int PP = 6; __VA_ARGS__; } \
+    case 7: { constexpr int PP = 7; __VA_ARGS__; } \
+    case 8: { constexpr int PP = 8; __VA_ARGS__; } \
+  }
+
+}  // namespace
+
+aabft_status launch_bound(const aabft_config *cfg, const aabft_encoded *enc, double *eps_col,
+                          double *sig_col, double *eps_row, double *sig_row, cudaStream_t st) {
+  const BoundParams bp = make_bound_params(cfg);
+  const int64_t n = (cfg->M / cfg->bs) * cfg->N + cfg->M * (cfg->N / cfg->bs);
+  const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, 148 * 16));
+  AABFT_P_SWITCH(cfg->p, {
+    bound_kernel<PP><<<grid, 256, 0, st>>>(cfg->M, cfg->N, cfg->bs, bp, enc->topA_val,
+                                           enc->topA_idx, enc->topB_val, enc->topB_idx, eps_col,
+                                           sig_col, eps_row, sig_row);
+    next_launch();
+    return check_launch("aabft_bound");
+  });
+  set_error("p out of range");
+  return AABFT_EINVAL;
+}
+
+aabft_status launch_check(const aabft_config *cfg, const aabft_encoded *enc,
+                          const aabft_product *prod, aabft_block_report *rep, aabft_counts *cnt,
+                          cudaStream_t st) {
+  const BoundParams bp = make_bound_params(cfg);
+  const CheckArgs a = make_args(cfg, enc, prod, rep, cnt);
+  if (cudaMemsetAsync(cnt, 0, sizeof(aabft_counts), st) != cudaSuccess)
+    return check_launch("aabft_check memset");
+  if (cfg->dtype == AABFT_F64) {
+    AABFT_P_SWITCH(cfg->p, return (run_check<double, PP>(cfg, a, bp, st)));
+  } else {
+    AABFT_P_SWITCH(cfg->p, return (run_check<float, PP>(cfg, a, bp, st)));
+  }
+  set_error("p out of range");
+  return AABFT_EINVAL;
+}
+
+aabft_status launch_correct(const aabft_config *cfg, const aabft_encoded *enc,
+                            const aabft_product *prod, aabft_block_report *rep,
+                            aabft_counts *cnt, cudaStream_t st) {
+  const BoundParams bp = make_bound_params(cfg);
+  const CheckArgs a = make_args(cfg, enc, prod, rep, cnt);
+  if (cfg->dtype == AABFT_F64) {
+    AABFT_P_SWITCH(cfg->p, return (run_correct<double, PP>(cfg, a, bp, st)));
+  } else {
+    AABFT_P_SWITCH(cfg->p, return (run_correct<float, PP>(cfg, a, bp, st)));
+  }
+  set_error("p out of range");
+  return AABFT_EINVAL;
+}
+
+}  // namespace aabft

@@ -1,0 +1,262 @@
+// encode.cu -- step 1 of A-ABFT on sm_100a: partitioned checksum encoding fused with top-p
+// |value| selection (P:L313-317 steps 1a-1d; Alg 1), and the global top-p
+// reduction (step 3, P:L320 / P:L368).
+//
+// B200 design: HBM-bound streaming.  One thread owns one column of a
+// BS-row block of A, so the column checksum is a register running sum in ascending row order
+// (bit-identical to Eq 1 summed top -> bottom, reading R11) and every warp load is a
+// contiguous 256 B row segment.  The same pass stages |a| in padded shared memory where four
+// lanes per row keep register top-p lists over interleaved columns and merge them with two
+// xor-shuffles (warp-shuffle top-p).  B is the mirror image: a thread owns a column of B
+// (running top-p over k in registers) and the BS-wide row sums are taken from the staged
+// tile, one sequential thread per (row, block).  Partial top-p lists per chunk are reduced
+// by a warp-per-vector kernel that also computes the top-p of the checksum vectors.
+#include <algorithm>
+
+#include "common.cuh"
+
+namespace aabft {
+namespace {
+
+constexpr int kStrip = 32;  // rows staged per pass
+
+template <typename T>
+__device__ __forceinline__ T ldg(const T *p) { return __ldg(p); }
+
+// ---------------------------------------------------------------------------------- A
+// grid (chunks of 128 columns, M/bs block-rows); 128 threads.
+template <typename T, int P>
+__global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, int64_t lda,
+                                                       int64_t K, int bs, T *__restrict__ Acs,
+                                                       int64_t ld_acs, double *__restrict__ pv,
+                                                       int *__restrict__ pi, int nch) {
+  __shared__ double tile[kStrip][kEncAChunk + 4];  // |A| strip; stride 132 -> conflict-free
+  const int c = threadIdx.x;
+  const int chunk = blockIdx.x;
+  const int64_t I = blockIdx.y;
+  const int64_t k = (int64_t)chunk * kEncAChunk + c;
+  const bool kin = k < K;
+  const int r = c >> 2, q = c & 3;  // top-p role: row r of the strip, column phase q
+  T sum = T(0);
+  for (int r0 = 0; r0 < bs; r0 += kStrip) {
+    const int rows = min(kStrip, bs - r0);
+    const T *src = A + (I * bs + r0) * lda + k;
+    T vals[kStrip];
+#pragma unroll
+    for (int rr = 0; rr < kStrip; ++rr) vals[rr] = (rr < rows && kin) ? ldg(src + rr * lda) : T(0);
+#pragma unroll
+    for (int rr = 0; rr < kStrip; ++rr) {
+      if (rr < rows) {
+        sum = sum + vals[rr];  // Eq 1, ascending i (Alg 1 line "sum <- sum + Asub[i][tid]")
+        tile[rr][c] = fabs((double)vals[rr]);
+      }
+    }
+    __syncthreads();
+    double v[P];
+    int ix[P];
+    tp_init<P>(v, ix);
+    if (r < rows) {
+#pragma unroll 4
+      for (int cc = q; cc < kEncAChunk; cc += 4) {
+        const int64_t kk = (int64_t)chunk * kEncAChunk + cc;
+        if (kk < K) tp_insert<P>(v, ix, tile[r][cc], (int)kk);
+      }
+    }
+    tp_shfl_merge<P>(v, ix, 1);
+    tp_shfl_merge<P>(v, ix, 2);
+    if (r < rows && q == 0) {
+      const int64_t row = I * bs + r0 + r;
+      double *dv = pv + (row * nch + chunk) * P;
+      int *di = pi + (row * nch + chunk) * P;
+#pragma unroll
+      for (int s = 0; s < P; ++s) { dv[s] = v[s]; di[s] = ix[s]; }
+    }
+    __syncthreads();
+  }
+  if (kin) Acs[I * ld_acs + k] = sum;
+}
+
+// ---------------------------------------------------------------------------------- B
+// grid (column chunks of NC, row chunks of kEncBChunk); NC threads (NC = max(128, bs)).
+template <typename T, int P, int NC>
+__global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, int64_t ldb,
+                                                      int64_t K, int64_t N, int bs,
+                                                      T *__restrict__ Bcs, int64_t ld_bcs,
+                                                      double *__restrict__ pv,
+                                                      int *__restrict__ pi, int nch) {
+  constexpr int SB = (NC * sizeof(T) > 1024) ? 16 : kStrip;  // strip rows (smem <= 48 KiB)
+  __shared__ T tile[SB][NC + 1];  // odd stride -> conflict-free per-row sequential reads
+  const int c = threadIdx.x;
+  const int64_t j = (int64_t)blockIdx.x * NC + c;
+  const bool jin = j < N;
+  const int kc = blockIdx.y;
+  const int64_t kbeg = (int64_t)kc * kEncBChunk;
+  const int64_t kend = K < kbeg + kEncBChunk ? K : kbeg + kEncBChunk;
+  const int nblk = NC / bs;  // checksum blocks covered by this CTA
+  double v[P];
+  int ix[P];
+  tp_init<P>(v, ix);
+  for (int64_t k0 = kbeg; k0 < kend; k0 += SB) {
+    const int rows = (int)(kend - k0 < SB ? kend - k0 : SB);
+    const T *src = B + k0 * ldb + j;
+    T vals[SB];
+#pragma unroll
+    for (int rr = 0; rr < SB; ++rr) vals[rr] = (rr < rows && jin) ? ldg(src + rr * ldb) : T(0);
+#pragma unroll
+    for (int rr = 0; rr < SB; ++rr) {
+      if (rr < rows) {
+        tile[rr][c] = vals[rr];
+        if (jin) tp_insert<P>(v, ix, fabs((double)vals[rr]), (int)(k0 + rr));
+      }
+    }
+    __syncthreads();
+    // Eq 2 row checksums: one thread per (row, block), sequential ascending j
+    for (int task = c; task < SB * nblk; task += NC) {
+      const int rr = task % SB, jb = task / SB;
+      const int64_t J = (int64_t)blockIdx.x * nblk + jb;
+      if (rr < rows && J * bs < N) {
+        T s = T(0);
+        for (int jj = 0; jj < bs; ++jj) s = s + tile[rr][jb * bs + jj];
+        Bcs[(k0 + rr) * ld_bcs + J] = s;
+      }
+    }
+    __syncthreads();
+  }
+  if (jin) {
+    double *dv = pv + (j * nch + kc) * P;
+    int *di = pi + (j * nch + kc) * P;
+#pragma unroll
+    for (int s = 0; s < P; ++s) { dv[s] = v[s]; di[s] = ix[s]; }
+  }
+}
+
+// ---------------------------------------------------------------------------------- step 3
+// One warp per vector: data rows of A / data cols of B merge their per-chunk partial lists;
+// checksum rows of Acs / checksum cols of Bcs are scanned directly.
+template <typename T, int P>
+__global__ void __launch_bounds__(256) topp_reduce_kernel(
+    int64_t M, int64_t N, int64_t K, int bs, const double *__restrict__ pva,
+    const int *__restrict__ pia, int ncha, const double *__restrict__ pvb,
+    const int *__restrict__ pib, int nchb, const T *__restrict__ Acs, int64_t ld_acs,
+    const T *__restrict__ Bcs, int64_t ld_bcs, double *__restrict__ topA_v,
+    int *__restrict__ topA_i, double *__restrict__ topB_v, int *__restrict__ topB_i, int do_a,
+    int do_b) {
+  const int lane = threadIdx.x & 31;
+  const int64_t w = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
+  const int64_t nA = do_a ? M + M / bs : 0;
+  const int64_t nB = do_b ? N + N / bs : 0;
+  if (w >= nA + nB) return;
+  double v[P];
+  int ix[P];
+  tp_init<P>(v, ix);
+  double *ov;
+  int *oi;
+  if (w < nA) {
+    if (w < M) {
+      const double *sv = pva + w * ncha * P;
+      const int *si = pia + w * ncha * P;
+      for (int e = lane; e < ncha * P; e += 32) tp_insert<P>(v, ix, sv[e], si[e]);
+    } else {
+      const T *row = Acs + (w - M) * ld_acs;
+      for (int64_t k = lane; k < K; k += 32) tp_insert<P>(v, ix, fabs((double)row[k]), (int)k);
+    }
+    ov = topA_v + w * P;
+    oi = topA_i + w * P;
+  } else {
+    const int64_t u = w - nA;
+    if (u < N) {
+      const double *sv = pvb + u * nchb * P;
+      const int *si = pib + u * nchb * P;
+      for (int e = lane; e < nchb * P; e += 32) tp_insert<P>(v, ix, sv[e], si[e]);
+    } else {
+      const T *col = Bcs + (u - N);
+      for (int64_t k = lane; k < K; k += 32)
+        tp_insert<P>(v, ix, fabs((double)col[k * ld_bcs]), (int)k);
+    }
+    ov = topB_v + u * P;
+    oi = topB_i + u * P;
+  }
+#pragma unroll
+  for (int m = 16; m >= 1; m >>= 1) tp_shfl_merge<P>(v, ix, m);
+  if (lane == 0) {
+#pragma unroll
+    for (int s = 0; s < P; ++s) { ov[s] = v[s]; oi[s] = ix[s]; }
+  }
+}
+
+template <typename T, int P>
+aabft_status run_encode(const aabft_config *cfg, const T *A, int64_t lda, const T *B,
+                        int64_t ldb, const aabft_encoded *out, void *ws, cudaStream_t st) {
+  const int64_t M = cfg->M, N = cfg->N, K = cfg->K;
+  const int bs = cfg->bs;
+  const int ncha = (int)enc_a_chunks(K), nchb = (int)enc_b_chunks(K);
+  char *w = static_cast<char *>(ws);
+  double *pva = reinterpret_cast<double *>(w);
+  w += ((size_t)M * ncha * P * 8 + 255) / 256 * 256;
+  int *pia = reinterpret_cast<int *>(w);
+  w += ((size_t)M * ncha * P * 4 + 255) / 256 * 256;
+  double *pvb = reinterpret_cast<double *>(w);
+  w += ((size_t)N * nchb * P * 8 + 255) / 256 * 256;
+  int *pib = reinterpret_cast<int *>(w);
+  if (A) {
+    dim3 grid(ncha, (unsigned)(M / bs));
+    encode_a_kernel<T, P><<<grid, 128, 0, st>>>(A, lda, K, bs, static_cast<T *>(out->Acs),
+                                                out->ld_acs, pva, pia, ncha);
+    next_launch();
+  }
+  if (B) {
+    const int NC = std::max(128, bs);
+    dim3 grid((unsigned)((N + NC - 1) / NC), nchb);
+    if (NC == 128)
+      encode_b_kernel<T, P, 128><<<grid, 128, 0, st>>>(B, ldb, K, N, bs, static_cast<T *>(out->Bcs),
+                                                       out->ld_bcs, pvb, pib, nchb);
+    else
+      encode_b_kernel<T, P, 256><<<grid, 256, 0, st>>>(B, ldb, K, N, bs, static_cast<T *>(out->Bcs),
+                                                       out->ld_bcs, pvb, pib, nchb);
+    next_launch();
+  }
+  const int64_t nvec = (A ? M + M / bs : 0) + (B ? N + N / bs : 0);
+  topp_reduce_kernel<T, P><<<(unsigned)((nvec + 7) / 8), 256, 0, st>>>(
+      M, N, K, bs, pva, pia, ncha, pvb, pib, nchb, static_cast<const T *>(out->Acs), out->ld_acs,
+      static_cast<const T *>(out->Bcs), out->ld_bcs, out->topA_val, out->topA_idx,
+      out->topB_val, out->topB_idx, A != nullptr, B != nullptr);
+  next_launch();
+  return check_launch("aabft_encode");
+}
+
+template <typename T>
+aabft_status dispatch_p(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
+                        int64_t ldb, const aabft_encoded *out, void *ws, cudaStream_t st) {
+  const T *a = static_cast<const T *>(A);
+  const T *b = static_cast<const T *>(B);
+  switch (cfg->p) {
+    case 1: return run_encode<T, 1>(cfg, a, lda, b, ldb, out, ws, st);
+    case 2: return run_encode<T, 2>(cfg, a, lda, b, ldb, out, ws, st);
+    case 3: return run_encode<T, 3>(cfg, a, lda, b, ldb, out, ws, st);
+    case 4: return run_encode<T, 4>(cfg, a, lda, b, ldb, out, ws, st);
+    case 5: return run_encode<T, 5>(cfg, a, lda, b, ldb, out, ws, st);
+    case 6: return run_encode<T, 6>(cfg, a, lda, b, ldb, out, ws, st);
+    case 7: return run_encode<T, 7>(cfg, a, lda, b, ldb, out, ws, st);
+    case 8: return run_encode<T, 8>(cfg, a, lda, b, ldb, out, ws, st);
+  }
+  set_error("p=%d out of range", cfg->p);
+  return AABFT_EINVAL;
+}
+
+}  // namespace
+
+size_t encode_ws_bytes(const aabft_config *cfg) {
+  const size_t p = (size_t)cfg->p;
+  const size_t ncha = (size_t)enc_a_chunks(cfg->K), nchb = (size_t)enc_b_chunks(cfg->K);
+  auto r = [](size_t b) { return (b + 255) / 256 * 256; };
+  return r(cfg->M * ncha * p * 8) + r(cfg->M * ncha * p * 4) + r(cfg->N * nchb * p * 8) +
+         r(cfg->N * nchb * p * 4);
+}
+
+aabft_status launch_encode(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
+                           int64_t ldb, const aabft_encoded *out, void *ws, cudaStream_t st) {
+  if (cfg->dtype == AABFT_F64) return dispatch_p<double>(cfg, A, lda, B, ldb, out, ws, st);
+  return dispatch_p<float>(cfg, A, lda, B, ldb, out, ws, st);
+}
+
+}  // namespace aabft

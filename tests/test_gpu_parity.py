@@ -1,0 +1,365 @@
+"""GPU parity: the sm_100a path (through the C ABI) against the CPU oracle, element by element.
+
+Bars (north_star / SURVEY §8(c)):
+  * Acs, Bcs, top-p values and indices, eps/sigma: bit-identical (sequential encode order).
+  * C, Ccol, Crow: |gpu - oracle| / (|A||B|) <= 1e-13 (FP64, DMMA order differs from the
+    sequential oracle) ; FP32 FFMA accumulates in the oracle's order -> bit-identical.
+  * Clean runs: zero CRITICAL, identical block verdicts.
+  * Faults outside 2x the bound: identical verdicts; located and corrected.
+"""
+import numpy as np
+import pytest
+
+import synth
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+TD = {np.float64: torch.float64, np.float32: torch.float32}
+
+
+@pytest.fixture(scope="module")
+def P():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_dsn_braunhw14_b200 import api
+    return api
+
+
+def gen(recipe, r, c, seed, mid, dtype=np.float64, **kw):
+    return synth.generate(recipe, r, c, seed=seed, matrix_id=mid, dtype=dtype, **kw)
+
+
+def to_dev(X):
+    """Row-major device copy whose pitch is a multiple of 16 bytes (ABI alignment rule)."""
+    X = np.ascontiguousarray(X)
+    r, c = X.shape
+    q = 16 // X.itemsize
+    ld = (c + q - 1) // q * q
+    buf = torch.zeros(r, ld, dtype=TD[X.dtype.type], device="cuda")
+    buf[:, :c] = torch.from_numpy(X).cuda()
+    return buf[:, :c]
+
+
+def host(t):
+    return t.detach().cpu().numpy()
+
+
+def norm_err(G, O, A, B):
+    denom = np.abs(A).astype(np.float64) @ np.abs(B).astype(np.float64)
+    denom[denom == 0] = 1.0
+    return float(np.max(np.abs(G.astype(np.float64) - O.astype(np.float64)) / denom))
+
+
+def xor_val(v, mask, dtype):
+    ut = np.uint64 if dtype == np.float64 else np.uint32
+    a = np.array([v], dtype=dtype).view(ut) ^ ut(mask)
+    with np.errstate(all="ignore"):
+        return float(a.view(dtype)[0])
+
+
+def run_both(P, orc, M, N, K, bs, p, dtype=np.float64, recipe="uniform", faults=(), seed=1,
+             correct=True, q=8):
+    A = gen(recipe, M, K, seed, 0, dtype, q=q)
+    B = gen(recipe, K, N, seed, 1, dtype, q=q)
+    plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p)
+    res = plan.run(to_dev(A), to_dev(B), faults=list(faults), correct=correct)
+    torch.cuda.synchronize()
+    o = orc.protected_matmul(A, B, bs=bs, p=p, faults=list(faults), do_correct=correct)
+    return A, B, plan, res, o
+
+
+SHAPES = [
+    # M, N, K, bs, p  (ragged: not multiples of the 128 tiles / 16-deep k-tiles)
+    (128, 128, 128, 32, 2),
+    (192, 320, 200, 64, 2),
+    (64, 96, 37, 8, 3),
+    (256, 256, 300, 256, 1),
+    (8, 8, 16, 8, 8),
+    (384, 128, 1000, 128, 4),
+]
+
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+@pytest.mark.parametrize("shape", SHAPES)
+def test_encode_bit_exact(P, orc, dtype, shape):
+    M, N, K, bs, p = shape
+    A = gen("uniform", M, K, 3, 0, dtype)
+    B = gen("wide", K, N, 3, 1, dtype)
+    plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p)
+    plan.encode(to_dev(A), to_dev(B))
+    torch.cuda.synchronize()
+    enc = orc.encode(A, B, bs, p)
+    assert np.array_equal(host(plan.Acs), enc["Acs"])
+    assert np.array_equal(host(plan.Bcs), enc["Bcs"])
+    assert np.array_equal(host(plan.topA_val), enc["topA"][0])
+    assert np.array_equal(host(plan.topA_idx), enc["topA"][1])
+    assert np.array_equal(host(plan.topB_val), enc["topB"][0])
+    assert np.array_equal(host(plan.topB_idx), enc["topB"][1])
+
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_encode_ties_integer_data(P, orc, dtype):
+    """Many equal |values|: the tie rule (lowest index) must match exactly."""
+    M, N, K, bs, p = 64, 64, 300, 16, 4
+    A = gen("integer", M, K, 5, 0, dtype, q=2)
+    B = gen("integer", K, N, 5, 1, dtype, q=2)
+    plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p)
+    plan.encode(to_dev(A), to_dev(B))
+    torch.cuda.synchronize()
+    enc = orc.encode(A, B, bs, p)
+    assert np.array_equal(host(plan.topA_idx), enc["topA"][1])
+    assert np.array_equal(host(plan.topB_idx), enc["topB"][1])
+    assert np.array_equal(host(plan.topA_val), enc["topA"][0])
+
+
+@pytest.mark.parametrize("fma_model", [1, 0])
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_bound_bit_exact(P, orc, dtype, fma_model):
+    M, N, K, bs, p = 192, 256, 333, 64, 2
+    A = gen("uniform100", M, K, 4, 0, dtype)
+    B = gen("uniform", K, N, 4, 1, dtype)
+    plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p, fma_model=fma_model)
+    plan.encode(to_dev(A), to_dev(B))
+    b = plan.bound()
+    torch.cuda.synchronize()
+    enc = orc.encode(A, B, bs, p)
+    o = orc.bounds_all(M, N, K, bs, p, enc["topA"], enc["topB"], t=orc.default_t(dtype),
+                       fma_model=fma_model)
+    for k in ("eps_col", "sig_col", "eps_row", "sig_row"):
+        assert np.array_equal(host(b[k]), o[k]), k
+
+
+@pytest.mark.parametrize("shape", SHAPES)
+def test_gemm_parity_f64(P, orc, shape):
+    M, N, K, bs, p = shape
+    A, B, plan, res, o = run_both(P, orc, M, N, K, bs, p)
+    enc = o["enc"]
+    assert norm_err(host(res.C), o["C"], A, B) <= 1e-13
+    assert norm_err(host(res.Ccol), o["Ccol"], enc["Acs"], B) <= 1e-13
+    assert norm_err(host(res.Crow), o["Crow"], A, enc["Bcs"]) <= 1e-13
+
+
+@pytest.mark.parametrize("shape", SHAPES)
+def test_gemm_parity_f32_bit_exact(P, orc, shape):
+    M, N, K, bs, p = shape
+    A, B, plan, res, o = run_both(P, orc, M, N, K, bs, p, dtype=np.float32, recipe="wide")
+    enc = o["enc"]
+    assert norm_err(host(res.C), o["C"], A, B) <= 1e-5
+    assert np.array_equal(host(res.C), o["C"])
+    assert np.array_equal(host(res.Ccol), o["Ccol"])
+    assert np.array_equal(host(res.Crow), o["Crow"])
+
+
+def test_gemm_plain_same_family(P, orc):
+    M, N, K = 256, 384, 520
+    for dtype in (np.float64, np.float32):
+        A = gen("uniform", M, K, 9, 0, dtype)
+        B = gen("uniform", K, N, 9, 1, dtype)
+        plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=64, p=2)
+        dA, dB = to_dev(A), to_dev(B)
+        plan.run(dA, dB)
+        Cp = P.gemm_plain(dA, dB)
+        torch.cuda.synchronize()
+        assert torch.equal(Cp, plan.C)  # identical data tiles -> identical bits
+        assert norm_err(host(Cp), orc.gemm(A, B), A, B) <= (1e-13 if dtype == np.float64 else 1e-5)
+
+
+@pytest.mark.parametrize("dtype,recipe", [(np.float64, "uniform"), (np.float64, "positive"),
+                                          (np.float64, "wide"), (np.float32, "uniform"),
+                                          (np.float32, "wide"), (np.float64, "integer")])
+def test_clean_run_verdicts(P, orc, dtype, recipe):
+    M, N, K, bs, p = 256, 192, 512, 64, 2
+    A, B, plan, res, o = run_both(P, orc, M, N, K, bs, p, dtype=dtype, recipe=recipe)
+    rep = res.reports()
+    cnt = res.counts()
+    assert cnt["checks_critical"] == 0 and o["check"].counts[7] == 0
+    assert np.all(rep["status"] == 0)
+    assert np.array_equal(rep["status"], o["check"].status)
+    assert cnt["blocks"] == (M // bs) * (N // bs) == cnt["clean"]
+    assert cnt["checks_rounding"] + cnt["checks_tolerable"] == (M // bs) * N + M * (N // bs)
+    assert cnt["max_ratio"] < 0.9
+    if recipe == "integer":
+        assert cnt["max_ratio"] == 0.0 and cnt["checks_rounding"] == o["check"].counts[5]
+
+
+def _fault_set(orc, A, B, bs, p, rng, dtype, n_per_mag=1):
+    """One fault per block: additive magnitudes r * max(eps_col, eps_row) across the band and
+    exponent/sign XOR flips."""
+    M, K = A.shape
+    N = B.shape[1]
+    enc = orc.encode(A, B, bs, p)
+    b = orc.bounds_all(M, N, K, bs, p, enc["topA"], enc["topB"], t=orc.default_t(dtype))
+    faults, labels = [], []
+    mags = [2.0 ** -8, 2.0 ** -4, 2.0 ** -2, 2.0 ** 2, 2.0 ** 5, 2.0 ** 12]
+    nI, nJ = M // bs, N // bs
+    n = 0
+    for I in range(nI):
+        for J in range(nJ):
+            i = I * bs + int(rng.integers(bs))
+            j = J * bs + int(rng.integers(bs))
+            lo = min(b["eps_col"][I, j], b["eps_row"][i, J])
+            hi = max(b["eps_col"][I, j], b["eps_row"][i, J])
+            kind = n % 8
+            n += 1
+            if kind < len(mags):
+                r = mags[kind] * (1 if rng.integers(2) else -1)
+                add = float(r * hi)
+                faults.append(dict(row=i, col=j, site=2, add=add))
+                labels.append("detect" if abs(add) > 2 * hi else ("silent" if abs(add) < 0.5 * lo else "band"))
+            elif kind == 6:
+                bit = 63 if dtype == np.float64 else 31
+                faults.append(dict(row=i, col=j, site=0, xor_mask=1 << bit))
+                labels.append("xor")
+            else:
+                bit = int(rng.integers(52, 63)) if dtype == np.float64 else int(rng.integers(23, 31))
+                faults.append(dict(row=i, col=j, site=0, xor_mask=1 << bit))
+                labels.append("xor")
+    return faults, labels
+
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_fault_verdicts_outside_band(P, orc, dtype):
+    M, N, K, bs, p = 512, 512, 256, 64, 2
+    rng = np.random.default_rng(42)
+    A = gen("uniform", M, K, 11, 0, dtype)
+    B = gen("uniform", K, N, 11, 1, dtype)
+    faults, labels = _fault_set(orc, A, B, bs, p, rng, dtype)
+    plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p)
+    dA, dB = to_dev(A), to_dev(B)
+    clean = host(plan.run(dA, dB).C).copy()
+    res = plan.run(dA, dB, faults=faults)
+    torch.cuda.synchronize()
+    rep = res.reports()
+    o = orc.protected_matmul(A, B, bs=bs, p=p, faults=faults)
+    ost = o["check"].status
+    Cg = host(res.C)
+    nchk = 0
+    for f, lab in zip(faults, labels):
+        I, J = f["row"] // bs, f["col"] // bs
+        g, og = rep["status"][I, J], ost[I, J]
+        clean_v = clean[f["row"], f["col"]]
+        if lab == "detect":
+            assert g == 1 and og == 1, (f, g, og)
+        elif lab == "silent":
+            assert g == 0 and og == 0, (f, g, og)
+        elif lab == "xor":
+            e = abs(xor_val(clean_v, f["xor_mask"], dtype) - clean_v)
+            if not np.isfinite(e) or e > 1e-3:
+                assert g == 1 and og == 1, (f, g, og)
+        if g == 1:
+            tol = 1e-12 if dtype == np.float64 else 1e-3
+            assert abs(Cg[f["row"], f["col"]] - clean_v) <= tol * max(1.0, abs(clean_v))
+        if lab != "band":
+            assert g == og, (f, lab, g, og)
+            nchk += 1
+    assert nchk > len(faults) // 2
+    # untouched elements are bit-identical to the clean run
+    mask = np.ones_like(Cg, bool)
+    for f in faults:
+        mask[f["row"], f["col"]] = False
+    assert np.array_equal(Cg[mask], clean[mask])
+
+
+def test_accumulator_fault_site1(P, orc):
+    M, N, K, bs, p = 256, 256, 512, 64, 2
+    A = gen("uniform", M, K, 12, 0)
+    B = gen("uniform", K, N, 12, 1)
+    plan = P.ProtectedGemm(M, N, K, dtype=torch.float64, bs=bs, p=p)
+    dA, dB = to_dev(A), to_dev(B)
+    clean = host(plan.run(dA, dB).C).copy()
+    faults = [dict(row=70, col=130, site=1, k_step=200, xor_mask=1 << 61),
+              dict(row=5, col=7, site=1, k_step=0, xor_mask=1 << 62),
+              dict(row=200, col=250, site=1, k_step=511, xor_mask=1 << 63)]
+    res = plan.run(dA, dB, faults=faults)
+    torch.cuda.synchronize()
+    rep = res.reports()
+    for f in faults:
+        assert rep["status"][f["row"] // bs, f["col"] // bs] == 1
+    assert np.allclose(host(res.C), clean, rtol=0, atol=1e-12)
+
+
+def test_checksum_faults_checksum_only(P, orc):
+    M, N, K, bs, p = 256, 256, 256, 64, 2
+    A = gen("uniform", M, K, 13, 0)
+    B = gen("uniform", K, N, 13, 1)
+    plan = P.ProtectedGemm(M, N, K, dtype=torch.float64, bs=bs, p=p)
+    dA, dB = to_dev(A), to_dev(B)
+    clean = host(plan.run(dA, dB).C).copy()
+    faults = [dict(row=M + 1, col=100, site=2, add=1.0),      # Ccol row 1
+              dict(row=10, col=N + 2, site=0, xor_mask=1 << 62)]  # Crow col 2
+    res = plan.run(dA, dB, faults=faults)
+    torch.cuda.synchronize()
+    rep = res.reports()
+    assert rep["status"][1, 100 // bs] == 2 and rep["status"][0, 2] == 2
+    assert res.counts()["checksum_only"] == 2
+    assert np.array_equal(host(res.C), clean)
+
+
+def test_multi_fault_block_uncorrectable(P, orc):
+    M, N, K, bs, p = 128, 128, 128, 64, 2
+    A = gen("uniform", M, K, 14, 0)
+    B = gen("uniform", K, N, 14, 1)
+    faults = [dict(row=3, col=4, site=2, add=5.0), dict(row=9, col=20, site=2, add=-3.0)]
+    A_, B_, plan, res, o = run_both(P, orc, M, N, K, bs, p, faults=faults, seed=14)
+    rep = res.reports()
+    assert rep["status"][0, 0] == 3 == o["check"].status[0, 0]
+    assert res.counts()["uncorrectable"] == 1
+
+
+def test_host_entry_point_e2e(P, orc):
+    """aabft_protected_gemm_host: host buffers in, corrected C + counts out."""
+    import ctypes as C
+    from paper_conf_dsn_braunhw14_b200 import _abi
+    M, N, K, bs = 256, 128, 200, 64
+    A = gen("uniform", M, K, 15, 0)
+    B = gen("uniform", K, N, 15, 1)
+    cfg = _abi.Config(0, bs, M, N, K, 2, 0, 3.0, 1, 0)
+    L = _abi.lib()
+    nbytes = L.aabft_host_arena_bytes(C.byref(cfg))
+    arena = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    Ch = np.zeros((M, N))
+    cnt = _abi.Counts()
+    st = L.aabft_protected_gemm_host(C.byref(cfg), A.ctypes.data, B.ctypes.data, Ch.ctypes.data,
+                                     C.addressof(cnt), arena.data_ptr(), nbytes,
+                                     torch.cuda.current_stream().cuda_stream)
+    _abi.ok(st, "aabft_protected_gemm_host")
+    assert norm_err(Ch, orc.gemm(A, B), A, B) <= 1e-13
+    assert cnt.n[0] == (M // bs) * (N // bs) == cnt.n[1] and cnt.n[7] == 0
+
+
+def test_full_size_c2_sampled(P, orc):
+    """BASELINE configs[1]: 4096^3 FP64, BS 64, the bench launch configuration.  The oracle
+    checks sampled rows / columns / blocks one by one."""
+    M = N = K = 4096
+    bs, p = 64, 2
+    A = gen("uniform", M, K, 1, 0)
+    B = gen("uniform", K, N, 2, 1)
+    plan = P.ProtectedGemm(M, N, K, dtype=torch.float64, bs=bs, p=p)
+    res = plan.run(to_dev(A), to_dev(B))
+    torch.cuda.synchronize()
+    cnt = res.counts()
+    assert cnt["blocks"] == 4096 and cnt["clean"] == 4096 and cnt["checks_critical"] == 0
+    assert cnt["max_ratio"] < 0.5
+    rng = np.random.default_rng(0)
+    tav, tai = host(plan.topA_val), host(plan.topA_idx)
+    tbv, tbi = host(plan.topB_val), host(plan.topB_idx)
+    Acs, Bcs, C = host(plan.Acs), host(plan.Bcs), host(res.C)
+    for i in rng.integers(0, M, 16):
+        v, ix = orc.topp_vector(A[i], p)
+        assert np.array_equal(tav[i], v) and np.array_equal(tai[i], ix)
+    for j in rng.integers(0, N, 16):
+        v, ix = orc.topp_vector(np.ascontiguousarray(B[:, j]), p)
+        assert np.array_equal(tbv[j], v) and np.array_equal(tbi[j], ix)
+    rows = rng.integers(0, M, 8)
+    assert norm_err(C[rows], orc.gemm(A[rows], B), A[rows], B) <= 1e-13
+    for (I, J) in [(0, 0), (63, 63), (17, 42), (40, 3)]:
+        Ab = A[I * bs:(I + 1) * bs]
+        Bb = np.ascontiguousarray(B[:, J * bs:(J + 1) * bs])
+        ob = orc.protected_matmul(Ab, Bb, bs=bs, p=p)
+        assert np.array_equal(Acs[I], ob["enc"]["Acs"][0])
+        assert np.array_equal(Bcs[:, J], ob["enc"]["Bcs"][:, 0])
+        assert np.array_equal(tav[M + I], ob["enc"]["topA"][0][bs])
+        assert np.array_equal(tbv[N + J], ob["enc"]["topB"][0][bs])
+        assert ob["check"].status[0, 0] == res.reports()["status"][I, J] == 0
+        assert norm_err(C[I * bs:(I + 1) * bs, J * bs:(J + 1) * bs], ob["C"], Ab, Bb) <= 1e-13
