@@ -147,8 +147,9 @@ typedef struct {
   double add;
 } aabft_fault; /* 48 bytes */
 
-/* Bytes of device workspace needed by aabft_encode / aabft_gemm / aabft_check (one buffer
- * serves all three; 256-byte aligned).  Returns 0 on an invalid config. */
+/* Bytes of device workspace needed by aabft_encode / aabft_gemm / aabft_gemm_plain /
+ * aabft_check (one buffer serves all of them; 256-byte aligned; contents need no
+ * initialisation).  Returns 0 on an invalid config. */
 size_t aabft_workspace_bytes(const aabft_config *cfg);
 
 /* Step 1 (Alg 1).  A (lda >= K) or B (ldb >= N) may be NULL to encode only the
@@ -173,9 +174,11 @@ aabft_status aabft_gemm(const aabft_config *cfg, const void *A, int64_t lda, con
                         const aabft_fault *faults, int32_t nfaults, void *ws, size_t ws_bytes,
                         void *stream);
 
-/* Unprotected C = A.B with the same kernel family (overhead denominator). */
+/* Unprotected C = A.B with the same kernel family and scheduler (overhead denominator).
+ * ws: device workspace of aabft_workspace_bytes(cfg) bytes (split-K partials). */
 aabft_status aabft_gemm_plain(const aabft_config *cfg, const void *A, int64_t lda,
-                              const void *B, int64_t ldb, void *C, int64_t ldc, void *stream);
+                              const void *B, int64_t ldb, void *C, int64_t ldc, void *ws,
+                              size_t ws_bytes, void *stream);
 
 /* Step 3 (Alg 2; Eq 4-6).  Writes (M/bs)*(N/bs) reports and zeroes then fills
  * *counts (device).  Reference sums are sequential ascending in double (reading R11/R12). */

@@ -93,7 +93,7 @@ def lib():
         L.aabft_bound.argtypes = [pc, C.POINTER(Encoded), vp, vp, vp, vp, vp]
         L.aabft_gemm.argtypes = [pc, vp, i64, vp, i64, C.POINTER(Encoded), C.POINTER(Product), vp,
                                  i32, vp, sz, vp]
-        L.aabft_gemm_plain.argtypes = [pc, vp, i64, vp, i64, vp, i64, vp]
+        L.aabft_gemm_plain.argtypes = [pc, vp, i64, vp, i64, vp, i64, vp, sz, vp]
         L.aabft_check.argtypes = [pc, C.POINTER(Encoded), C.POINTER(Product), vp, vp, vp, sz, vp]
         L.aabft_correct.argtypes = [pc, C.POINTER(Encoded), C.POINTER(Product), vp, vp, vp]
         L.aabft_protected_gemm_host.argtypes = [pc, vp, vp, vp, vp, vp, sz, vp]

@@ -224,17 +224,26 @@ def protected_matmul(A, B, *, bs: int = 64, p: int = 2, omega: float = 3.0, t: i
     return plan.run(A, B, faults=faults, correct=correct)
 
 
+_plain_ws = {}
+
+
 def gemm_plain(A, B, out=None, stream=None):
-    """Unprotected C = A @ B with the same kernel family (overhead denominator)."""
+    """Unprotected C = A @ B with the same kernel family and scheduler (overhead denominator)."""
     M, K = A.shape
     N = B.shape[1]
     dt = A.dtype
+    if M % 8 or N % 8:
+        raise ValueError("gemm_plain: M and N must be multiples of 8")
     if out is None:
         out = torch.empty(M, _pad_ld(N, dt), dtype=dt, device=A.device)
     cfg = Config(_dtype_code(dt), 8, M, N, K, 1, 0, 3.0, 1, 0)  # bs=8: validation only
-    if M % 8 or N % 8:
-        raise ValueError("gemm_plain: M and N must be multiples of 8")
+    wsb = int(lib().aabft_workspace_bytes(C.byref(cfg)))
+    key = (A.device, wsb)
+    if key not in _plain_ws:
+        _plain_ws.clear()
+        _plain_ws[key] = torch.empty(wsb, dtype=torch.uint8, device=A.device)
+    ws = _plain_ws[key]
     ok(lib().aabft_gemm_plain(C.byref(cfg), A.data_ptr(), A.stride(0), B.data_ptr(), B.stride(0),
-                              out.data_ptr(), out.stride(0), _stream_ptr(stream)),
-       "aabft_gemm_plain")
+                              out.data_ptr(), out.stride(0), ws.data_ptr(), wsb,
+                              _stream_ptr(stream)), "aabft_gemm_plain")
     return out[:, :N]

@@ -11,8 +11,6 @@
 
 namespace aabft {
 
-size_t encode_ws_bytes(const aabft_config *cfg);
-
 namespace {
 thread_local char g_err[512] = "";
 std::atomic<int64_t> g_launches{0};
@@ -103,6 +101,13 @@ static aabft_status device_ok() {
 }
 
 // rows of a row-major operand fed to TMA / vector loads: base 16-B aligned, pitch 16-B multiple
+static size_t gemm_ws_bytes(const aabft_config *c) {
+  return c->dtype == AABFT_F64 ? gemm_f64_ws_bytes() : 0;
+}
+static void *gemm_ws(const aabft_config *c, void *ws) {
+  return static_cast<char *>(ws) + r256(encode_ws_bytes(c));
+}
+
 static bool pitch_ok(const aabft_config *c, const void *p, int64_t ld) {
   return aligned16(p) && ((size_t)ld * elem_size(c)) % 16 == 0;
 }
@@ -123,7 +128,8 @@ extern "C" {
 
 size_t aabft_workspace_bytes(const aabft_config *cfg) {
   if (validate(cfg) != AABFT_OK) return 0;
-  return r256(encode_ws_bytes(cfg)) + 256;
+  // [encode partial top-p lists][FP64 GEMM split-K partials + flags]
+  return r256(encode_ws_bytes(cfg)) + r256(gemm_ws_bytes(cfg)) + 256;
 }
 
 aabft_status aabft_encode(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
@@ -168,9 +174,13 @@ aabft_status aabft_bound(const aabft_config *cfg, const aabft_encoded *enc, doub
 static aabft_status gemm_common(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
                                 int64_t ldb, const aabft_encoded *enc, const aabft_product *out,
                                 const aabft_fault *faults, int32_t nfaults, bool plain,
-                                void *stream) {
+                                void *ws, size_t ws_bytes, void *stream) {
   aabft_status s = validate(cfg);
   if (s != AABFT_OK) return s;
+  if (!ws || ws_bytes < aabft_workspace_bytes(cfg)) {
+    set_error("workspace too small: need %zu bytes", aabft_workspace_bytes(cfg));
+    return AABFT_EWORKSPACE;
+  }
   if (!A || !B || !out || !out->C) { set_error("gemm: A, B, C required"); return AABFT_EINVAL; }
   if (lda < cfg->K || ldb < cfg->N || out->ldc < cfg->N) { set_error("gemm: lda >= K, ldb >= N, ldc >= N required"); return AABFT_EINVAL; }
   if (!pitch_ok(cfg, A, lda) || !pitch_ok(cfg, B, ldb) || !aligned16(out->C)) {
@@ -191,7 +201,7 @@ static aabft_status gemm_common(const aabft_config *cfg, const void *A, int64_t 
   }
   if ((s = device_ok()) != AABFT_OK) return s;
   if (cfg->dtype == AABFT_F64)
-    return launch_gemm_f64(cfg, A, lda, B, ldb, enc, out, plain ? nullptr : faults, plain ? 0 : nfaults, plain, (cudaStream_t)stream);
+    return launch_gemm_f64(cfg, A, lda, B, ldb, enc, out, plain ? nullptr : faults, plain ? 0 : nfaults, plain, gemm_ws(cfg, ws), (cudaStream_t)stream);
   return launch_gemm_f32(cfg, A, lda, B, ldb, enc, out, plain ? nullptr : faults, plain ? 0 : nfaults, plain, (cudaStream_t)stream);
 }
 
@@ -200,19 +210,18 @@ aabft_status aabft_gemm(const aabft_config *cfg, const void *A, int64_t lda, con
                         const aabft_fault *faults, int32_t nfaults, void *ws, size_t ws_bytes,
                         void *stream) {
   AABFT_GUARD_BEGIN
-  (void)ws;
-  (void)ws_bytes;
-  return gemm_common(cfg, A, lda, B, ldb, enc, out, faults, nfaults, false, stream);
+  return gemm_common(cfg, A, lda, B, ldb, enc, out, faults, nfaults, false, ws, ws_bytes, stream);
   AABFT_GUARD_END
 }
 
 aabft_status aabft_gemm_plain(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
-                              int64_t ldb, void *C, int64_t ldc, void *stream) {
+                              int64_t ldb, void *C, int64_t ldc, void *ws, size_t ws_bytes,
+                              void *stream) {
   AABFT_GUARD_BEGIN
   aabft_product out{};
   out.C = C;
   out.ldc = ldc;
-  return gemm_common(cfg, A, lda, B, ldb, nullptr, &out, nullptr, 0, true, stream);
+  return gemm_common(cfg, A, lda, B, ldb, nullptr, &out, nullptr, 0, true, ws, ws_bytes, stream);
   AABFT_GUARD_END
 }
 

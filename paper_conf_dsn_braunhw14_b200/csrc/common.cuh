@@ -46,7 +46,9 @@ aabft_status launch_bound(const aabft_config *cfg, const aabft_encoded *enc, dou
 aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda,
                              const void *B, int64_t ldb, const aabft_encoded *enc,
                              const aabft_product *out, const aabft_fault *faults,
-                             int32_t nfaults, bool plain, cudaStream_t st);
+                             int32_t nfaults, bool plain, void *ws, cudaStream_t st);
+size_t encode_ws_bytes(const aabft_config *cfg);
+size_t gemm_f64_ws_bytes();
 aabft_status launch_gemm_f32(const aabft_config *cfg, const void *A, int64_t lda,
                              const void *B, int64_t ldb, const aabft_encoded *enc,
                              const aabft_product *out, const aabft_fault *faults,

@@ -3,35 +3,49 @@
 //
 // B200 design:
 //  * tcgen05.mma has no f64 kind, so the FP64 tensor path is warp-level
-//    mma.sync.aligned.m16n8k4.row.col.f64 (SASS DMMA); measured issue ceiling 37.0 TFLOP/s
-//    (profiles/r01_step0_pipes.jsonl) vs 34 TFLOP/s for DFMA.
-//  * One elected thread issues TMA (cp.async.bulk.tensor) into a 4-stage shared-memory ring
-//    guarded by full/empty mbarriers; 8 MMA warps (2 x 4, 64 x 32 warp tiles) read swizzled
-//    fragments with conflict-free 64-bit LDS and issue 16 DMMAs per k4-step.
-//    A tiles use the 128B swizzle (box 16 k x 128 rows), B tiles are 16 boxes of 8 columns x
-//    16 k with the 64B swizzle -- both make the m16n8k4 fragment loads bank-conflict free.
-//  * One launch computes all three products of Eq 3 with partitioned checksums: C = A.B,
-//    Ccol = Acs.B (checksum rows as their own tiles), Crow = A.Bcs (checksum columns as
-//    their own tiles).  The corner Acs.Bcs is never formed (reading R17).
-//  * Fault hooks: a CTA copies the faults that hit its tile into shared memory; site 1 XORs
-//    the accumulator after the k-tile containing k_step, sites 0/2 act on the stored value.
+//    mma.sync.aligned.m16n8k4.row.col.f64 (SASS DMMA.8x8x4); measured issue ceiling
+//    37.0 TFLOP/s (profiles/r01_step0_pipes.jsonl) vs 34 TFLOP/s for DFMA.
+//  * Persistent CTAs (one per SM, 8 MMA warps, 255-register budget).  Work = all tiles of the
+//    three products of Eq 3 with partitioned checksums, each the same amount of MMA work:
+//       type 0  C    = A.B     128 x 128 tiles
+//       type 1  Ccol = Acs.B    64 x 256 tiles  (checksum rows: M/BS of them)
+//       type 2  Crow = A.Bcs   256 x  64 tiles  (checksum cols: N/BS of them)
+//    so the checksum work costs its ideal 2/BS share instead of half-empty 128 x 128 tiles.
+//    The corner Acs.Bcs is never formed (reading R17).
+//  * Scheduling: full waves are data-parallel (tile c + w*G for CTA c; grouped raster keeps
+//    a wave's A/B panels L2-resident); the ragged remainder is split along K (stream-K) so
+//    every SM gets the same number of k-tiles -- no wave-quantisation tail.  Split tiles are
+//    reduced deterministically: the CTA holding k-chunk 0 adds the partials of the following
+//    CTAs in ascending k order.
+//  * TMA (cp.async.bulk.tensor) fills a 4-stage ring guarded by full mbarriers; the last warp
+//    to release a stage refills it (across tile boundaries).  A tiles use the 128B swizzle
+//    (box 16 k x 64/128 rows), B tiles are boxes of 8 columns x 16 k with the 64B swizzle;
+//    with the k-permutation below every 64-bit fragment LDS is bank-conflict free.
+//  * Fault hooks (Alg 3): site 1 XORs the accumulator after the k-tile containing k_step (in
+//    a split tile: the partial accumulator of the CTA that owns that k-tile); sites 0/2 act
+//    on the stored value.
 #include <cudaTypedefs.h>
+
+#include <algorithm>
 
 #include "common.cuh"
 
 namespace aabft {
+
+size_t gemm_f64_ws_bytes();
+
 namespace {
 
-constexpr int BM = 128, BN = 128, BK = 16, STAGES = 4;
-constexpr int NCW = 8;                     // MMA warps (2 x 4)
-constexpr int THREADS = NCW * 32;          // 256: 2 warps / SMSP -> up to 255 registers
-constexpr int A_BYTES = BM * BK * 8;       // 16 KiB
-constexpr int B_BYTES = BK * BN * 8;       // 16 KiB
-constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+constexpr int BK = 16, STAGES = 4;
+constexpr int NCW = 8;                     // MMA warps
+constexpr int THREADS = NCW * 32;          // 2 warps / SMSP -> up to 255 registers
+constexpr int STAGE_BYTES = 40 * 1024;     // max over tile types of A + B bytes
 constexpr int MAXF = 16;                   // faults per tile kept in smem
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/ +
-                           MAXF * (int)sizeof(aabft_fault) + 16;
+                           MAXF * (int)sizeof(aabft_fault) + 64;
 constexpr int GROUP_M = 8;
+constexpr int kMaxCtas = 160;              // >= SM count; sizes the split-K partial slots
+constexpr int ACC = 64;                    // accumulators per thread
 
 struct GemmArgs {
   int64_t M, N, K, Mcs, Ncs;
@@ -41,18 +55,63 @@ struct GemmArgs {
   int64_t ld_ccol;
   double *Crow;
   int64_t ld_crow;
-  int64_t n0, n1, n2;       // tiles of type 0 (data), 1 (column checksums), 2 (row checksums)
-  int tm0, tn0, tm1, tn2;   // tile grid dims
-  int nk;
+  int tm0, tn0, tm1, tn1, tm2, tn2;   // tile grids of the three types
+  int64_t n0, n1, n2, ntiles;
+  int nk;                             // k-tiles per tile
+  int waves;                          // data-parallel waves
+  int64_t sk_iters;                   // k-tiles in the stream-K remainder
+  double *partials;                   // [kMaxCtas][ACC][THREADS]
+  int *flags;                         // [kMaxCtas]
   const aabft_fault *faults;
   int nfaults;
 };
 
-__device__ __forceinline__ int swz128(int r, int k) {  // A tile [128 rows][16 k] doubles
-  return r * 16 + ((((k >> 1) ^ (r & 7)) << 1) | (k & 1));
+struct Tile {
+  int type;
+  int64_t m0, n0;
+};
+
+__device__ __forceinline__ Tile tile_of(const GemmArgs &a, int64_t t) {
+  Tile r;
+  if (t < a.n0) {
+    r.type = 0;
+    const int64_t group = (int64_t)GROUP_M * a.tn0;
+    const int64_t g = t / group;
+    const int first_m = (int)(g * GROUP_M);
+    const int gm = min(a.tm0 - first_m, GROUP_M);
+    const int64_t in = t % group;
+    r.m0 = (int64_t)(first_m + (int)(in % gm)) * 128;
+    r.n0 = (in / gm) * 128;
+  } else if (t < a.n0 + a.n1) {
+    t -= a.n0;
+    r.type = 1;
+    r.m0 = (t / a.tn1) * 64;
+    r.n0 = (t % a.tn1) * 256;
+  } else {
+    t -= a.n0 + a.n1;
+    r.type = 2;
+    r.m0 = (t / a.tn2) * 256;
+    r.n0 = (t % a.tn2) * 64;
+  }
+  return r;
 }
-__device__ __forceinline__ int swz64(int k, int n) {   // B sub-box [16 k][8 n] doubles
-  return k * 8 + ((((n >> 1) ^ ((k >> 1) & 3)) << 1) | (n & 1));
+
+// the CTA's j-th k-tile: (tile index, k-tile index)
+__device__ __forceinline__ void iter_of(const GemmArgs &a, int j, int64_t sk0, int64_t &tile,
+                                        int &kt) {
+  const int64_t dp = (int64_t)a.waves * a.nk;
+  if (j < dp) {
+    tile = blockIdx.x + (j / a.nk) * gridDim.x;
+    kt = (int)(j % a.nk);
+  } else {
+    const int64_t it = sk0 + (j - dp);
+    tile = (int64_t)a.waves * gridDim.x + it / a.nk;
+    kt = (int)(it % a.nk);
+  }
+}
+
+__device__ __forceinline__ int64_t sk_begin(const GemmArgs &a, int64_t c) {
+  return a.sk_iters * c / gridDim.x;
 }
 
 __device__ __forceinline__ void dmma(double (&c)[4], double a0, double a1, double b) {
@@ -72,201 +131,303 @@ __global__ void __launch_bounds__(THREADS, 1)
                     const __grid_constant__ CUtensorMap tmAcs,
                     const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmBcs, const GemmArgs args) {
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
-                                              ~uintptr_t(1023));
+  extern __shared__ __align__(16) uint8_t smem_raw[];
+  // 1024-B aligned ring (swizzle atoms); offset applied to the __shared__ array itself so the
+  // compiler keeps the shared address space (32-bit LDS, not generic 64-bit loads)
+  const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
+  uint8_t *smem = smem_raw + pad;
   uint64_t *full = reinterpret_cast<uint64_t *>(smem + STAGES * STAGE_BYTES);
-  uint64_t *empty = full + STAGES;
-  int *s_nf = reinterpret_cast<int *>(empty + STAGES);
+  uint32_t *s_rel = reinterpret_cast<uint32_t *>(full + STAGES);  // per-stage release counters
+  int *s_nf = reinterpret_cast<int *>(s_rel + STAGES);
+  int *s_flag = s_nf + 1;
   aabft_fault *s_f = reinterpret_cast<aabft_fault *>(smem + STAGES * STAGE_BYTES + 256);
+  static_assert(8 * STAGES + 4 * STAGES + 4 * 8 <= 256, "bookkeeping fits");
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int g = lane >> 2, tig = lane & 3;
+  const int wm = warp >> 2, wn = warp & 3;
 
-  // ---- tile decode (type 0 grouped raster for L2 reuse)
-  int64_t bid = blockIdx.x;
-  int type, tm, tn;
-  if (bid < args.n0) {
-    type = 0;
-    const int64_t group = (int64_t)GROUP_M * args.tn0;
-    const int64_t g = bid / group;
-    const int first_m = (int)(g * GROUP_M);
-    const int gm = min(args.tm0 - first_m, GROUP_M);
-    const int64_t in = bid % group;
-    tm = first_m + (int)(in % gm);
-    tn = (int)(in / gm);
-  } else if (bid < args.n0 + args.n1) {
-    type = 1;
-    bid -= args.n0;
-    tm = (int)(bid / args.tn0);
-    tn = (int)(bid % args.tn0);
-  } else {
-    type = 2;
-    bid -= args.n0 + args.n1;
-    tm = (int)(bid / args.tn2);
-    tn = (int)(bid % args.tn2);
-  }
-  const int m0 = tm * BM, n0 = tn * BN;
-  const int64_t rows_valid = type == 1 ? args.Mcs : args.M;
-  const int64_t cols_valid = type == 2 ? args.Ncs : args.N;
+  // this CTA's k-tile sequence: its data-parallel tiles, then its stream-K slice
+  const int64_t sk0 = sk_begin(args, blockIdx.x), sk1 = sk_begin(args, blockIdx.x + 1);
+  const int njobs = args.waves * args.nk + (int)(sk1 - sk0);
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&empty[s], NCW);
+      s_rel[s] = 0;
     }
-    *s_nf = 0;
     fence_barrier_init();
   }
   __syncthreads();
 
-  // Producer role: thread 0 issues TMA.  Prologue fills the ring; afterwards, at the top of
-  // k-tile kt it refills the slot consumed at kt-1 once all 8 warps released it (empty
-  // barrier), so the refill lags the slowest warp by one k-tile and never blocks the MMAs of
-  // the stages already resident.  (A dedicated 9th producer warp would cap registers at 168:
-  // 3 warps on one SMSP.)
-  const CUtensorMap *ta = type == 1 ? &tmAcs : &tmA;
-  const CUtensorMap *tb = type == 2 ? &tmBcs : &tmB;
-  auto issue = [&](int kt) {
-    const int s = kt % STAGES;
-    uint8_t *sa = smem + s * STAGE_BYTES;
-    uint8_t *sb = sa + A_BYTES;
-    mbar_arrive_expect_tx(&full[s], STAGE_BYTES);
-    tma_load_2d(sa, ta, &full[s], kt * BK, m0);
-#pragma unroll
-    for (int b = 0; b < BN / 8; ++b) tma_load_2d(sb + b * 1024, tb, &full[s], n0 + b * 8, kt * BK);
+  // TMA producer.  Jobs are issued strictly in order (the refill of job j + STAGES happens
+  // only after every warp released job j), so a shared-memory cursor holds the decoded next
+  // job; advancing it is O(1) except at tile boundaries.  The issuing WARP spreads the box
+  // copies over its lanes (one cp.async.bulk.tensor per lane).
+  int *cur = s_flag + 1;  // [0] next job, [1] tile, [2] kt, [3] type, [4] m0, [5] n0
+  auto decode = [&](int jn) {
+    int64_t t;
+    int kt;
+    iter_of(args, jn, sk0, t, kt);
+    const Tile tl = tile_of(args, t);
+    cur[0] = jn; cur[1] = (int)t; cur[2] = kt; cur[3] = tl.type; cur[4] = (int)tl.m0;
+    cur[5] = (int)tl.n0;
   };
-  if (threadIdx.x == 0) {
-    tma_prefetch_desc(ta);
-    tma_prefetch_desc(tb);
-    for (int kt = 0; kt < STAGES && kt < args.nk; ++kt) issue(kt);
-  }
-
-  // ================= consumers
-  const int wm = warp >> 2, wn = warp & 3;  // 2 x 4 warps, 64 x 32 warp tiles
-  const int g = lane >> 2, tig = lane & 3;
-
-  // collect faults that hit this tile (C_fc coordinates -> tile-local)
-  int nf = 0;
-  if (args.nfaults > 0) {
-    for (int f = threadIdx.x; f < args.nfaults; f += NCW * 32) {
-      const aabft_fault ft = args.faults[f];
-      int64_t r = ft.row, c = ft.col;
-      bool hit;
-      if (type == 0) hit = r < args.M && c < args.N;
-      else if (type == 1) { hit = r >= args.M && c < args.N; r -= args.M; }
-      else { hit = c >= args.N && r < args.M; c -= args.N; }
-      if (hit && r >= m0 && r < m0 + BM && c >= n0 && c < n0 + BN) {
-        const int slot = atomicAdd(s_nf, 1);
-        if (slot < MAXF) {
-          aabft_fault loc = ft;
-          loc.row = r - m0;
-          loc.col = c - n0;
-          s_f[slot] = loc;
+  auto issue_warp = [&]() {  // called by all 32 lanes of one warp, convergent
+    const int jn = cur[0], kt = cur[2], type = cur[3], m0 = cur[4], n0 = cur[5];
+    const int s = jn % STAGES;
+    uint8_t *sa = smem + s * STAGE_BYTES;
+    const int k = kt * BK;
+    if (lane == 0) mbar_arrive_expect_tx(&full[s], type == 0 ? 32 * 1024 : 40 * 1024);
+    __syncwarp();
+    if (type == 0) {
+      if (lane < 16) tma_load_2d(sa + 16 * 1024 + lane * 1024, &tmB, &full[s], n0 + lane * 8, k);
+      else if (lane == 16) tma_load_2d(sa, &tmA, &full[s], k, m0);
+    } else if (type == 1) {
+      tma_load_2d(sa + 8 * 1024 + lane * 1024, &tmB, &full[s], n0 + lane * 8, k);
+      if (lane == 0) tma_load_2d(sa, &tmAcs, &full[s], k, m0);
+    } else {
+      if (lane < 8) tma_load_2d(sa + 32 * 1024 + lane * 1024, &tmBcs, &full[s], n0 + lane * 8, k);
+      else if (lane < 10) tma_load_2d(sa + (lane - 8) * 16 * 1024, &tmA, &full[s], k, m0 + (lane - 8) * 128);
+    }
+    __syncwarp();
+    if (lane == 0) {  // advance the cursor
+      if (jn + 1 < njobs) {
+        if (kt + 1 < args.nk && (jn + 1) != args.waves * args.nk) {
+          cur[0] = jn + 1;
+          cur[2] = kt + 1;
+        } else {
+          decode(jn + 1);
         }
       }
     }
-    __syncthreads();
-    nf = min(*s_nf, MAXF);
+    __syncwarp();
+  };
+  if (warp == 0) {
+    if (lane == 0) {
+      tma_prefetch_desc(&tmA);
+      tma_prefetch_desc(&tmB);
+      tma_prefetch_desc(&tmAcs);
+      tma_prefetch_desc(&tmBcs);
+      if (njobs > 0) decode(0);
+    }
+    __syncwarp();
+    for (int jn = 0; jn < STAGES && jn < njobs; ++jn) issue_warp();
   }
 
   double acc[4][4][4];
-#pragma unroll
-  for (int i = 0; i < 4; ++i)
-#pragma unroll
-    for (int j = 0; j < 4; ++j)
-#pragma unroll
-      for (int q = 0; q < 4; ++q) acc[i][j][q] = 0.0;
+  int j = 0;
+  while (j < njobs) {
+    // ---------------- segment = consecutive k-tiles of one tile
+    int64_t tile;
+    int kt0;
+    iter_of(args, j, sk0, tile, kt0);
+    const Tile tl = tile_of(args, tile);
+    const int seg_len = (int)(args.nk - kt0 < njobs - j ? args.nk - kt0 : njobs - j);
+    const int kt_end = kt0 + seg_len;  // exclusive
 
-  for (int kt = 0; kt < args.nk; ++kt) {
-    const int s = kt % STAGES;
-    if (threadIdx.x == 0 && kt >= 1 && kt - 1 + STAGES < args.nk) {
-      mbar_wait(&empty[(kt - 1) % STAGES], ((kt - 1) / STAGES) & 1);
-      issue(kt - 1 + STAGES);
+    int arow, bbox0, boff;
+    int64_t rbase, cbase;
+    if (tl.type == 0) {
+      arow = wm * 64; bbox0 = wn * 4; boff = 16 * 1024;
+      rbase = tl.m0 + wm * 64; cbase = tl.n0 + wn * 32;
+    } else if (tl.type == 1) {
+      arow = 0; bbox0 = wm * 16 + wn * 4; boff = 8 * 1024;
+      rbase = tl.m0; cbase = tl.n0 + wm * 128 + wn * 32;
+    } else {
+      const int rb = wm + 2 * (wn >> 1);
+      arow = rb * 64; bbox0 = (wn & 1) * 4; boff = 32 * 1024;
+      rbase = tl.m0 + rb * 64; cbase = tl.n0 + (wn & 1) * 32;
     }
-    mbar_wait(&full[s], (kt / STAGES) & 1);
-    const double *sa = reinterpret_cast<const double *>(smem + s * STAGE_BYTES);
-    const double *sb = reinterpret_cast<const double *>(smem + s * STAGE_BYTES + A_BYTES);
+    // Fragment addressing.  The mma k index (= tig) of k4-step ks maps to the k-tile column
+    //   k = pi(ks, tig) = (tig&1) | (ks&1)<<1 | ((tig>>1)^(ks>>1))<<2 | (tig>>1)<<3
+    // (a bijection of [0,16); the same permutation for A and B leaves the product unchanged).
+    // With the 128B-swizzled A tile and the 64B-swizzled B boxes every half-warp of a 64-bit
+    // LDS touches 16 distinct 8-byte bank slots (conflict-free: 2 wavefronts).
+    uint32_t offA[4], offB[4];
 #pragma unroll
-    for (int ks = 0; ks < BK / 4; ++ks) {
-      const int k = ks * 4 + tig;
-      double a[4][2], b[4];
-#pragma unroll
-      for (int mt = 0; mt < 4; ++mt) {
-        const int r = wm * 64 + mt * 16 + g;
-        a[mt][0] = sa[swz128(r, k)];
-        a[mt][1] = sa[swz128(r + 8, k)];
+    for (int ks = 0; ks < 4; ++ks) {
+      const int k = (tig & 1) | ((ks & 1) << 1) | ((((tig >> 1) ^ (ks >> 1)) & 1) << 2) | ((tig >> 1) << 3);
+      offA[ks] = (uint32_t)(((arow + g) * 16 + ((((k >> 1) ^ g) << 1) | (k & 1))) * 8);
+      offB[ks] = (uint32_t)(boff + bbox0 * 1024 +
+                            (k * 8 + ((((g >> 1) ^ ((k >> 1) & 3)) << 1) | (g & 1))) * 8);
+    }
+
+    // faults that hit this tile (output coordinates of the tile's product)
+    int nf = 0;
+    if (args.nfaults > 0) {
+      __syncthreads();
+      if (threadIdx.x == 0) *s_nf = 0;
+      __syncthreads();
+      const int64_t rows = tl.type == 0 ? 128 : (tl.type == 1 ? 64 : 256);
+      const int64_t cols = tl.type == 0 ? 128 : (tl.type == 1 ? 256 : 64);
+      for (int f = threadIdx.x; f < args.nfaults; f += THREADS) {
+        aabft_fault ft = args.faults[f];
+        int64_t r = ft.row, c = ft.col;
+        int ftype;
+        if (r < args.M && c < args.N) ftype = 0;
+        else if (r >= args.M && c < args.N) { ftype = 1; r -= args.M; }
+        else if (c >= args.N && r < args.M) { ftype = 2; c -= args.N; }
+        else ftype = -1;
+        if (ftype == tl.type && r >= tl.m0 && r < tl.m0 + rows && c >= tl.n0 && c < tl.n0 + cols) {
+          const int slot = atomicAdd(s_nf, 1);
+          if (slot < MAXF) {
+            ft.row = r;
+            ft.col = c;
+            s_f[slot] = ft;
+          }
+        }
       }
+      __syncthreads();
+      nf = min(*s_nf, MAXF);
+    }
+
 #pragma unroll
-      for (int nt = 0; nt < 4; ++nt) b[nt] = sb[(wn * 4 + nt) * 128 + swz64(k, g)];
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int jj = 0; jj < 4; ++jj)
+#pragma unroll
+        for (int q = 0; q < 4; ++q) acc[i][jj][q] = 0.0;
+
+    for (int kt = kt0; kt < kt_end; ++kt, ++j) {
+      const int s = (int)(j % STAGES);
+      mbar_wait(&full[s], (uint32_t)((j / STAGES) & 1));
+      const uint8_t *st = smem + s * STAGE_BYTES;
+      double a[2][4][2], b[2][4];
+      auto load = [&](int buf, int ks) {
+#pragma unroll
+        for (int mt = 0; mt < 4; ++mt) {
+          a[buf][mt][0] = *reinterpret_cast<const double *>(st + offA[ks] + mt * 2048);
+          a[buf][mt][1] = *reinterpret_cast<const double *>(st + offA[ks] + mt * 2048 + 1024);
+        }
+#pragma unroll
+        for (int nt = 0; nt < 4; ++nt)
+          b[buf][nt] = *reinterpret_cast<const double *>(st + offB[ks] + nt * 1024);
+      };
+      load(0, 0);
+#pragma unroll
+      for (int ks = 0; ks < BK / 4; ++ks) {
+        if (ks + 1 < BK / 4) load((ks + 1) & 1, ks + 1);
+#pragma unroll
+        for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+          for (int nt = 0; nt < 4; ++nt)
+            dmma(acc[mt][nt], a[ks & 1][mt][0], a[ks & 1][mt][1], b[ks & 1][nt]);
+      }
+      // release the stage; the last of the 8 warps refills it with job j + STAGES
+      __syncwarp();
+      uint32_t prev = 0;
+      if (lane == 0) {
+        __threadfence_block();
+        prev = atomicAdd(&s_rel[s], 1u);
+      }
+      prev = __shfl_sync(0xffffffffu, prev, 0);
+      if (prev == (uint32_t)(NCW * (j / STAGES + 1) - 1) && j + STAGES < njobs) {
+        __threadfence_block();
+        fence_proxy_async();
+        issue_warp();
+      }
+      if (nf > 0) {  // Alg 3 errorVecAdd1 at k-tile granularity
+        for (int f = 0; f < nf; ++f) {
+          const aabft_fault ft = s_f[f];
+          if (ft.site != 1 || ft.k_step / BK != kt) continue;
+#pragma unroll
+          for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+            for (int nt = 0; nt < 4; ++nt)
+#pragma unroll
+              for (int q = 0; q < 4; ++q) {
+                const int64_t r = rbase + mt * 16 + g + (q >> 1) * 8;
+                const int64_t c = cbase + nt * 8 + tig * 2 + (q & 1);
+                if (r == ft.row && c == ft.col) acc[mt][nt][q] = xor_bits(acc[mt][nt][q], ft.xor_mask);
+              }
+        }
+      }
+    }
+
+    // ---------------- segment epilogue
+    const bool first = kt0 == 0, last = kt_end == args.nk;
+    if (!first) {
+      // contributor: park the partial accumulators, then signal the owner
+      double *slot = args.partials + (int64_t)blockIdx.x * ACC * THREADS + threadIdx.x;
 #pragma unroll
       for (int mt = 0; mt < 4; ++mt)
 #pragma unroll
-        for (int nt = 0; nt < 4; ++nt) dmma(acc[mt][nt], a[mt][0], a[mt][1], b[nt]);
+        for (int nt = 0; nt < 4; ++nt)
+#pragma unroll
+          for (int q = 0; q < 4; ++q) slot[((mt * 4 + nt) * 4 + q) * THREADS] = acc[mt][nt][q];
+      __threadfence();
+      __syncthreads();
+      if (threadIdx.x == 0) atomicExch(&args.flags[blockIdx.x], 1);
+      continue;
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[s]);
-    if (nf > 0) {  // Alg 3 errorVecAdd1 at k-tile granularity
+    if (!last) {
+      // owner of a split tile: add the partials of the following CTAs in ascending k order
+      const int64_t tile_it_end = (tile - (int64_t)args.waves * gridDim.x + 1) * args.nk;
+      for (int64_t c = blockIdx.x + 1; c < gridDim.x && sk_begin(args, c) < tile_it_end; ++c) {
+        if (sk_begin(args, c + 1) == sk_begin(args, c)) continue;  // empty slice: no partial
+        if (threadIdx.x == 0) {
+          while (atomicAdd(&args.flags[c], 0) == 0) __nanosleep(64);
+          atomicExch(&args.flags[c], 0);  // re-arm for the next launch
+          __threadfence();
+          *s_flag = 1;
+        }
+        __syncthreads();
+        const double *slot = args.partials + c * ACC * THREADS + threadIdx.x;
+#pragma unroll
+        for (int mt = 0; mt < 4; ++mt)
+#pragma unroll
+          for (int nt = 0; nt < 4; ++nt)
+#pragma unroll
+            for (int q = 0; q < 4; ++q)
+              acc[mt][nt][q] += __ldcg(slot + ((mt * 4 + nt) * 4 + q) * THREADS);
+        __syncthreads();
+      }
+    }
+    if (nf > 0) {
       for (int f = 0; f < nf; ++f) {
         const aabft_fault ft = s_f[f];
-        if (ft.site != 1 || ft.k_step / BK != kt) continue;
+        if (ft.site == 1) continue;
 #pragma unroll
         for (int mt = 0; mt < 4; ++mt)
 #pragma unroll
           for (int nt = 0; nt < 4; ++nt)
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
-              const int r = wm * 64 + mt * 16 + g + (q >> 1) * 8;
-              const int c = wn * 32 + nt * 8 + tig * 2 + (q & 1);
-              if (r == ft.row && c == ft.col) acc[mt][nt][q] = xor_bits(acc[mt][nt][q], ft.xor_mask);
+              const int64_t r = rbase + mt * 16 + g + (q >> 1) * 8;
+              const int64_t c = cbase + nt * 8 + tig * 2 + (q & 1);
+              if (r == ft.row && c == ft.col)
+                acc[mt][nt][q] = ft.site == 0 ? xor_bits(acc[mt][nt][q], ft.xor_mask)
+                                              : acc[mt][nt][q] + ft.add;
             }
       }
     }
-  }
-
-  // ================= epilogue: faults on the stored value, then masked 16-byte stores
-  if (nf > 0) {
-    for (int f = 0; f < nf; ++f) {
-      const aabft_fault ft = s_f[f];
-      if (ft.site == 1) continue;
+    double *out;
+    int64_t ld, rows_valid, cols_valid;
+    if (tl.type == 0) { out = args.C; ld = args.ldc; rows_valid = args.M; cols_valid = args.N; }
+    else if (tl.type == 1) { out = args.Ccol; ld = args.ld_ccol; rows_valid = args.Mcs; cols_valid = args.N; }
+    else { out = args.Crow; ld = args.ld_crow; rows_valid = args.M; cols_valid = args.Ncs; }
+    const bool vec_ok = (ld % 2 == 0) && ((reinterpret_cast<uintptr_t>(out) & 15) == 0);
 #pragma unroll
-      for (int mt = 0; mt < 4; ++mt)
+    for (int mt = 0; mt < 4; ++mt)
 #pragma unroll
-        for (int nt = 0; nt < 4; ++nt)
+      for (int h = 0; h < 2; ++h) {
+        const int64_t r = rbase + mt * 16 + g + h * 8;
+        if (r >= rows_valid) continue;
 #pragma unroll
-          for (int q = 0; q < 4; ++q) {
-            const int r = wm * 64 + mt * 16 + g + (q >> 1) * 8;
-            const int c = wn * 32 + nt * 8 + tig * 2 + (q & 1);
-            if (r == ft.row && c == ft.col)
-              acc[mt][nt][q] = ft.site == 0 ? xor_bits(acc[mt][nt][q], ft.xor_mask)
-                                            : acc[mt][nt][q] + ft.add;
+        for (int nt = 0; nt < 4; ++nt) {
+          const int64_t c = cbase + nt * 8 + tig * 2;
+          double *p = out + r * ld + c;
+          const double v0 = acc[mt][nt][h * 2], v1 = acc[mt][nt][h * 2 + 1];
+          if (c + 1 < cols_valid && vec_ok) {
+            *reinterpret_cast<double2 *>(p) = make_double2(v0, v1);
+          } else {
+            if (c < cols_valid) p[0] = v0;
+            if (c + 1 < cols_valid) p[1] = v1;
           }
-    }
-  }
-  double *out;
-  int64_t ld;
-  if (type == 0) { out = args.C; ld = args.ldc; }
-  else if (type == 1) { out = args.Ccol; ld = args.ld_ccol; }
-  else { out = args.Crow; ld = args.ld_crow; }
-  const bool vec_ok = (ld % 2 == 0) && ((reinterpret_cast<uintptr_t>(out) & 15) == 0);
-#pragma unroll
-  for (int mt = 0; mt < 4; ++mt)
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const int64_t r = m0 + wm * 64 + mt * 16 + g + h * 8;
-      if (r >= rows_valid) continue;
-#pragma unroll
-      for (int nt = 0; nt < 4; ++nt) {
-        const int64_t c = n0 + wn * 32 + nt * 8 + tig * 2;
-        double *p = out + r * ld + c;
-        const double v0 = acc[mt][nt][h * 2], v1 = acc[mt][nt][h * 2 + 1];
-        if (c + 1 < cols_valid && vec_ok) {
-          *reinterpret_cast<double2 *>(p) = make_double2(v0, v1);
-        } else {
-          if (c < cols_valid) p[0] = v0;
-          if (c + 1 < cols_valid) p[1] = v1;
         }
       }
-    }
+  }
 }
 
 PFN_cuTensorMapEncodeTiled_v12000 get_encoder() {
@@ -307,16 +468,24 @@ bool make_map(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer, 
 
 }  // namespace
 
+size_t gemm_f64_ws_bytes() {
+  return (size_t)kMaxCtas * ACC * THREADS * sizeof(double) + kMaxCtas * sizeof(int) + 256;
+}
+
 aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
                              int64_t ldb, const aabft_encoded *enc, const aabft_product *out,
-                             const aabft_fault *faults, int32_t nfaults, bool plain,
+                             const aabft_fault *faults, int32_t nfaults, bool plain, void *ws,
                              cudaStream_t st) {
-  static bool attr_set = false;
-  if (!attr_set) {
+  static int num_sms = 0;
+  if (!num_sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (cudaDeviceGetAttribute(&num_sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
+      return check_launch("gemm_f64 SM count");
     if (cudaFuncSetAttribute(gemm_f64_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              SMEM_BYTES) != cudaSuccess)
       return check_launch("gemm_f64 smem attribute");
-    attr_set = true;
+    num_sms = std::min(num_sms, kMaxCtas);
   }
   const int64_t M = cfg->M, N = cfg->N, K = cfg->K, bs = cfg->bs;
   GemmArgs a{};
@@ -328,32 +497,46 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
   a.ld_ccol = plain ? 0 : out->ld_ccol;
   a.Crow = plain ? nullptr : static_cast<double *>(out->Crow);
   a.ld_crow = plain ? 0 : out->ld_crow;
-  a.tm0 = (int)((M + BM - 1) / BM);
-  a.tn0 = (int)((N + BN - 1) / BN);
-  a.tm1 = plain ? 0 : (int)((a.Mcs + BM - 1) / BM);
-  a.tn2 = plain ? 0 : (int)((a.Ncs + BN - 1) / BN);
+  a.tm0 = (int)((M + 127) / 128);
+  a.tn0 = (int)((N + 127) / 128);
+  a.tm1 = plain ? 0 : (int)((a.Mcs + 63) / 64);
+  a.tn1 = (int)((N + 255) / 256);
+  a.tm2 = (int)((M + 255) / 256);
+  a.tn2 = plain ? 0 : (int)((a.Ncs + 63) / 64);
   a.n0 = (int64_t)a.tm0 * a.tn0;
-  a.n1 = (int64_t)a.tm1 * a.tn0;
-  a.n2 = (int64_t)a.tm0 * a.tn2;
+  a.n1 = (int64_t)a.tm1 * a.tn1;
+  a.n2 = (int64_t)a.tm2 * a.tn2;
+  a.ntiles = a.n0 + a.n1 + a.n2;
   a.nk = (int)((K + BK - 1) / BK);
+  const int64_t total = a.ntiles * a.nk;
+  const int grid = (int)std::min<int64_t>(num_sms, total);
+  // full data-parallel waves, keeping at least ~1/2 wave of tiles for the stream-K tail so
+  // every CTA's k-slice stays long enough to amortise its fixup
+  int waves = (int)(a.ntiles / grid);
+  if (waves > 0 && a.ntiles % grid != 0 && (a.ntiles % grid) * 2 < grid) waves -= 1;
+  a.waves = waves;
+  a.sk_iters = (a.ntiles - (int64_t)waves * grid) * a.nk;
+  a.partials = static_cast<double *>(ws);
+  a.flags = reinterpret_cast<int *>(static_cast<char *>(ws) + (size_t)kMaxCtas * ACC * THREADS * sizeof(double));
   a.faults = faults;
   a.nfaults = faults ? nfaults : 0;
 
   CUtensorMap tA, tAcs, tB, tBcs;
-  if (!make_map(&tA, A, K, M, lda, BK, BM, CU_TENSOR_MAP_SWIZZLE_128B)) return AABFT_EINVAL;
+  if (!make_map(&tA, A, K, M, lda, BK, 128, CU_TENSOR_MAP_SWIZZLE_128B)) return AABFT_EINVAL;
   if (!make_map(&tB, B, N, K, ldb, 8, BK, CU_TENSOR_MAP_SWIZZLE_64B)) return AABFT_EINVAL;
   if (plain) {
     tAcs = tA;
     tBcs = tB;
   } else {
-    if (!make_map(&tAcs, enc->Acs, K, a.Mcs, enc->ld_acs, BK, BM, CU_TENSOR_MAP_SWIZZLE_128B))
+    if (!make_map(&tAcs, enc->Acs, K, a.Mcs, enc->ld_acs, BK, 64, CU_TENSOR_MAP_SWIZZLE_128B))
       return AABFT_EINVAL;
     if (!make_map(&tBcs, enc->Bcs, a.Ncs, K, enc->ld_bcs, 8, BK, CU_TENSOR_MAP_SWIZZLE_64B))
       return AABFT_EINVAL;
   }
-  const int64_t tiles = a.n0 + a.n1 + a.n2;
-  if (tiles > 0) {
-    gemm_f64_kernel<<<(unsigned)tiles, THREADS, SMEM_BYTES, st>>>(tA, tAcs, tB, tBcs, a);
+  if (total > 0) {
+    if (a.sk_iters > 0 && cudaMemsetAsync(a.flags, 0, kMaxCtas * sizeof(int), st) != cudaSuccess)
+      return check_launch("gemm_f64 flag reset");
+    gemm_f64_kernel<<<grid, THREADS, SMEM_BYTES, st>>>(tA, tAcs, tB, tBcs, a);
     next_launch();
   }
   return check_launch("aabft_gemm(f64)");

@@ -107,7 +107,7 @@ def test_workspace_and_null_checks(L):
     # misaligned operand for the TMA GEMM
     prod = _abi.Product(16, 256, 16, 256, 16, 4)
     st = L.aabft_gemm(C.byref(cfg), 8, 256, 16, 256, C.byref(enc), C.byref(prod), None, 0, 16,
-                      1 << 20, None)
+                      1 << 40, None)
     assert st == 1 and b"aligned" in L.aabft_last_error()
     assert L.aabft_status_str(4).startswith(b"AABFT_EWORKSPACE")
     assert L.aabft_version().startswith(b"aabft-b200")

@@ -161,7 +161,9 @@ def test_gemm_plain_same_family(P, orc):
         plan.run(dA, dB)
         Cp = P.gemm_plain(dA, dB)
         torch.cuda.synchronize()
-        assert torch.equal(Cp, plan.C)  # identical data tiles -> identical bits
+        # same kernel family; the stream-K split of the ragged tail may differ between the
+        # two launches (different tile sets), so compare by tolerance, not bits
+        assert norm_err(host(Cp), host(plan.C), A, B) <= (1e-13 if dtype == np.float64 else 0)
         assert norm_err(host(Cp), orc.gemm(A, B), A, B) <= (1e-13 if dtype == np.float64 else 1e-5)
 
 
