@@ -11,7 +11,8 @@ import os
 import numpy as np
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libaabft.so")
+# AABFT_LIB selects an alternative build of the same library (tuning experiments only)
+LIB_PATH = os.environ.get("AABFT_LIB", os.path.join(HERE, "libaabft.so"))
 
 F64, F32 = 0, 1
 BLK_CLEAN, BLK_CORRECTED, BLK_CHECKSUM_ONLY, BLK_UNCORRECTABLE, BLK_SINGLE = 0, 1, 2, 3, 4

@@ -11,12 +11,13 @@ from concurrent.futures import ThreadPoolExecutor
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-OUT = os.path.join(HERE, "libaabft.so")
-OBJ = os.path.join(HERE, "build")
+OUT = os.environ.get("AABFT_BUILD_OUT", os.path.join(HERE, "libaabft.so"))
+OBJ = os.environ.get("AABFT_BUILD_OBJ", os.path.join(HERE, "build"))
 SOURCES = ["api.cu", "encode.cu", "check.cu", "gemm_f64.cu", "gemm_f32.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
-         "-Xcompiler", "-fPIC,-ffp-contract=off", "-Xptxas", "-v", "-I", os.path.join(HERE, "..", "include")]
+         "-Xcompiler", "-fPIC,-ffp-contract=off", "-Xptxas", "-v", "-I", os.path.join(HERE, "..", "include"),
+         *os.environ.get("AABFT_EXTRA_FLAGS", "").split()]
 
 
 def _stale(obj: str, deps) -> bool:

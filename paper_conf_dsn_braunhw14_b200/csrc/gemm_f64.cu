@@ -3,24 +3,24 @@
 //
 // B200 design:
 //  * tcgen05.mma has no f64 kind, so the FP64 tensor path is warp-level
-//    mma.sync.aligned.m16n8k4.row.col.f64 (SASS DMMA.8x8x4); measured issue ceiling
-//    37.0 TFLOP/s (profiles/r01_step0_pipes.jsonl) vs 34 TFLOP/s for DFMA.
-//  * Persistent CTAs (one per SM, 8 MMA warps, 255-register budget).  Work = all tiles of the
-//    three products of Eq 3 with partitioned checksums, each the same amount of MMA work:
-//       type 0  C    = A.B     128 x 128 tiles
-//       type 1  Ccol = Acs.B    64 x 256 tiles  (checksum rows: M/BS of them)
-//       type 2  Crow = A.Bcs   256 x  64 tiles  (checksum cols: N/BS of them)
-//    so the checksum work costs its ideal 2/BS share instead of half-empty 128 x 128 tiles.
-//    The corner Acs.Bcs is never formed (reading R17).
-//  * Scheduling: full waves are data-parallel (tile c + w*G for CTA c; grouped raster keeps
-//    a wave's A/B panels L2-resident); the ragged remainder is split along K (stream-K) so
-//    every SM gets the same number of k-tiles -- no wave-quantisation tail.  Split tiles are
-//    reduced deterministically: the CTA holding k-chunk 0 adds the partials of the following
-//    CTAs in ascending k order.
-//  * TMA (cp.async.bulk.tensor) fills a 4-stage ring guarded by full mbarriers; the last warp
-//    to release a stage refills it (across tile boundaries).  A tiles use the 128B swizzle
-//    (box 16 k x 64/128 rows), B tiles are boxes of 8 columns x 16 k with the 64B swizzle;
-//    with the k-permutation below every 64-bit fragment LDS is bank-conflict free.
+//    mma.sync.aligned.m16n8k4.row.col.f64 (SASS DMMA.8x8x4: 512 flop, one per 16 cycles per
+//    SM sub-partition; measured ceiling 37.0 TFLOP/s, profiles/r01_step0_pipes.jsonl).
+//  * The DMMA pipe is kept busy by many INDEPENDENT warps rather than big register tiles:
+//    64 x 64 CTA tiles, 4 MMA warps (2 x 2, 32 x 32 warp tiles, 128 registers) + 1 TMA
+//    producer warp, 3 CTAs per SM, each with its own ring -- a stall in one CTA never blocks
+//    another.
+//  * All three products of Eq 3 with partitioned checksums use the same 64 x 64 tile:
+//    C = A.B, Ccol = Acs.B (M/BS checksum rows), Crow = A.Bcs (N/BS checksum columns); the
+//    checksum work costs its ideal 2/BS share when M/BS, N/BS are multiples of 64.  The corner
+//    Acs.Bcs is never formed (reading R17).
+//  * Persistent scheduling: full waves are data-parallel (grouped raster keeps a wave's A/B
+//    panels L2-resident); the ragged remainder is split along K (stream-K) so every CTA gets
+//    the same number of k-tiles.  Split tiles are reduced deterministically: the CTA holding
+//    k-chunk 0 adds the partials of the following CTAs in ascending k order.
+//  * A dedicated producer warp per CTA streams TMA (cp.async.bulk.tensor) copies through a
+//    4-stage full/empty mbarrier ring (across tile boundaries), one box per lane.  A tiles use the 128B swizzle (box 16 k x 64 rows), B tiles are 8 boxes of 8
+//    columns x 16 k with the 64B swizzle; with the k-permutation below every 64-bit fragment
+//    LDS is bank-conflict free.
 //  * Fault hooks (Alg 3): site 1 XORs the accumulator after the k-tile containing k_step (in
 //    a split tile: the partial accumulator of the CTA that owns that k-tile); sites 0/2 act
 //    on the stored value.
@@ -32,20 +32,30 @@
 
 namespace aabft {
 
-size_t gemm_f64_ws_bytes();
-
 namespace {
 
-constexpr int BK = 16, STAGES = 4;
-constexpr int NCW = 8;                     // MMA warps
-constexpr int THREADS = NCW * 32;          // 2 warps / SMSP -> up to 255 registers
-constexpr int STAGE_BYTES = 40 * 1024;     // max over tile types of A + B bytes
-constexpr int MAXF = 16;                   // faults per tile kept in smem
-constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + 256 /*barriers*/ +
-                           MAXF * (int)sizeof(aabft_fault) + 64;
-constexpr int GROUP_M = 8;
-constexpr int kMaxCtas = 160;              // >= SM count; sizes the split-K partial slots
-constexpr int ACC = 64;                    // accumulators per thread
+#ifndef AABFT_F64_STAGES
+#define AABFT_F64_STAGES 4
+#endif
+#ifndef AABFT_F64_GROUP_M
+#define AABFT_F64_GROUP_M 16
+#endif
+constexpr int TILE = 64, BK = 16, STAGES = AABFT_F64_STAGES;
+constexpr int NCW = 4;                      // MMA warps per CTA (2 x 2)
+constexpr int THREADS = NCW * 32;           // MMA threads (named barrier 1)
+constexpr int CTA_THREADS = THREADS + 32;   // + 1 TMA producer warp
+constexpr int CTAS_PER_SM = 3;              // 15 warps / SM -> 128 registers each
+constexpr int MT = 2, NT = 4;               // m16 x n8 fragments per warp: 32 x 32 warp tile
+constexpr int A_BYTES = TILE * BK * 8;      // 8 KiB
+constexpr int B_BYTES = BK * TILE * 8;      // 8 KiB
+constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+constexpr int MAXF = 16;                    // faults per tile kept in smem
+constexpr int BOOK = 128;                   // barriers, counters, cursor
+constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + BOOK +
+                           MAXF * (int)sizeof(aabft_fault);
+constexpr int GROUP_M = AABFT_F64_GROUP_M;
+constexpr int kMaxCtas = 1024;              // >= resident CTAs; sizes the split-K partial slots
+constexpr int ACC = MT * NT * 4;            // accumulators per thread
 
 struct GemmArgs {
   int64_t M, N, K, Mcs, Ncs;
@@ -55,8 +65,8 @@ struct GemmArgs {
   int64_t ld_ccol;
   double *Crow;
   int64_t ld_crow;
-  int tm0, tn0, tm1, tn1, tm2, tn2;   // tile grids of the three types
-  int64_t n0, n1, n2, ntiles;
+  int tm0, tn0, tm1, tn2;             // tile grids: data tm0 x tn0, Ccol tm1 x tn0, Crow tm0 x tn2
+  int n0, n1, n2, ntiles;
   int nk;                             // k-tiles per tile
   int waves;                          // data-parallel waves
   int64_t sk_iters;                   // k-tiles in the stream-K remainder
@@ -67,51 +77,49 @@ struct GemmArgs {
 };
 
 struct Tile {
-  int type;
-  int64_t m0, n0;
+  int type, m0, n0;
 };
 
-__device__ __forceinline__ Tile tile_of(const GemmArgs &a, int64_t t) {
+__device__ __forceinline__ Tile tile_of(const GemmArgs &a, int t) {
   Tile r;
   if (t < a.n0) {
     r.type = 0;
-    const int64_t group = (int64_t)GROUP_M * a.tn0;
-    const int64_t g = t / group;
-    const int first_m = (int)(g * GROUP_M);
+    const int group = GROUP_M * a.tn0;
+    const int g = t / group;
+    const int first_m = g * GROUP_M;
     const int gm = min(a.tm0 - first_m, GROUP_M);
-    const int64_t in = t % group;
-    r.m0 = (int64_t)(first_m + (int)(in % gm)) * 128;
-    r.n0 = (in / gm) * 128;
+    const int in = t % group;
+    r.m0 = (first_m + in % gm) * TILE;
+    r.n0 = (in / gm) * TILE;
   } else if (t < a.n0 + a.n1) {
     t -= a.n0;
     r.type = 1;
-    r.m0 = (t / a.tn1) * 64;
-    r.n0 = (t % a.tn1) * 256;
+    r.m0 = (t / a.tn0) * TILE;
+    r.n0 = (t % a.tn0) * TILE;
   } else {
     t -= a.n0 + a.n1;
     r.type = 2;
-    r.m0 = (t / a.tn2) * 256;
-    r.n0 = (t % a.tn2) * 64;
+    r.m0 = (t / a.tn2) * TILE;
+    r.n0 = (t % a.tn2) * TILE;
   }
   return r;
 }
 
-// the CTA's j-th k-tile: (tile index, k-tile index)
-__device__ __forceinline__ void iter_of(const GemmArgs &a, int j, int64_t sk0, int64_t &tile,
-                                        int &kt) {
-  const int64_t dp = (int64_t)a.waves * a.nk;
-  if (j < dp) {
-    tile = blockIdx.x + (j / a.nk) * gridDim.x;
-    kt = (int)(j % a.nk);
-  } else {
-    const int64_t it = sk0 + (j - dp);
-    tile = (int64_t)a.waves * gridDim.x + it / a.nk;
-    kt = (int)(it % a.nk);
-  }
-}
-
 __device__ __forceinline__ int64_t sk_begin(const GemmArgs &a, int64_t c) {
   return a.sk_iters * c / gridDim.x;
+}
+
+// the CTA's j-th k-tile: (tile index, k-tile index)
+__device__ __forceinline__ void iter_of(const GemmArgs &a, int j, int64_t sk0, int &tile, int &kt) {
+  const int dp = a.waves * a.nk;
+  if (j < dp) {
+    tile = (int)blockIdx.x + (j / a.nk) * (int)gridDim.x;
+    kt = j % a.nk;
+  } else {
+    const int64_t it = sk0 + (j - dp);
+    tile = a.waves * (int)gridDim.x + (int)(it / a.nk);
+    kt = (int)(it % a.nk);
+  }
 }
 
 __device__ __forceinline__ void dmma(double (&c)[4], double a0, double a1, double b) {
@@ -122,11 +130,16 @@ __device__ __forceinline__ void dmma(double (&c)[4], double a0, double a1, doubl
       : "d"(a0), "d"(a1), "d"(b));
 }
 
+// barrier among the 4 MMA warps only (the producer warp never joins)
+__device__ __forceinline__ void mma_sync_bar() {
+  asm volatile("bar.sync 1, %0;" ::"n"(THREADS) : "memory");
+}
+
 __device__ __forceinline__ double xor_bits(double v, uint64_t m) {
   return __longlong_as_double(__double_as_longlong(v) ^ (long long)m);
 }
 
-__global__ void __launch_bounds__(THREADS, 1)
+__global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
     gemm_f64_kernel(const __grid_constant__ CUtensorMap tmA,
                     const __grid_constant__ CUtensorMap tmAcs,
                     const __grid_constant__ CUtensorMap tmB,
@@ -137,15 +150,14 @@ __global__ void __launch_bounds__(THREADS, 1)
   const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
   uint8_t *smem = smem_raw + pad;
   uint64_t *full = reinterpret_cast<uint64_t *>(smem + STAGES * STAGE_BYTES);
-  uint32_t *s_rel = reinterpret_cast<uint32_t *>(full + STAGES);  // per-stage release counters
-  int *s_nf = reinterpret_cast<int *>(s_rel + STAGES);
-  int *s_flag = s_nf + 1;
-  aabft_fault *s_f = reinterpret_cast<aabft_fault *>(smem + STAGES * STAGE_BYTES + 256);
-  static_assert(8 * STAGES + 4 * STAGES + 4 * 8 <= 256, "bookkeeping fits");
+  uint64_t *empty = full + STAGES;
+  int *s_nf = reinterpret_cast<int *>(empty + STAGES);
+  static_assert(16 * STAGES + 8 <= BOOK, "bookkeeping fits");
+  aabft_fault *s_f = reinterpret_cast<aabft_fault *>(smem + STAGES * STAGE_BYTES + BOOK);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int g = lane >> 2, tig = lane & 3;
-  const int wm = warp >> 2, wn = warp & 3;
+  const int wm = warp >> 1, wn = warp & 1;
 
   // this CTA's k-tile sequence: its data-parallel tiles, then its stream-K slice
   const int64_t sk0 = sk_begin(args, blockIdx.x), sk1 = sk_begin(args, blockIdx.x + 1);
@@ -154,113 +166,79 @@ __global__ void __launch_bounds__(THREADS, 1)
   if (threadIdx.x == 0) {
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&full[s], 1);
-      s_rel[s] = 0;
+      mbar_init(&empty[s], NCW);
     }
     fence_barrier_init();
   }
   __syncthreads();
 
-  // TMA producer.  Jobs are issued strictly in order (the refill of job j + STAGES happens
-  // only after every warp released job j), so a shared-memory cursor holds the decoded next
-  // job; advancing it is O(1) except at tile boundaries.  The issuing WARP spreads the box
-  // copies over its lanes (one cp.async.bulk.tensor per lane).
-  int *cur = s_flag + 1;  // [0] next job, [1] tile, [2] kt, [3] type, [4] m0, [5] n0
-  auto decode = [&](int jn) {
-    int64_t t;
-    int kt;
-    iter_of(args, jn, sk0, t, kt);
-    const Tile tl = tile_of(args, t);
-    cur[0] = jn; cur[1] = (int)t; cur[2] = kt; cur[3] = tl.type; cur[4] = (int)tl.m0;
-    cur[5] = (int)tl.n0;
-  };
-  auto issue_warp = [&]() {  // called by all 32 lanes of one warp, convergent
-    const int jn = cur[0], kt = cur[2], type = cur[3], m0 = cur[4], n0 = cur[5];
-    const int s = jn % STAGES;
-    uint8_t *sa = smem + s * STAGE_BYTES;
-    const int k = kt * BK;
-    if (lane == 0) mbar_arrive_expect_tx(&full[s], type == 0 ? 32 * 1024 : 40 * 1024);
-    __syncwarp();
-    if (type == 0) {
-      if (lane < 16) tma_load_2d(sa + 16 * 1024 + lane * 1024, &tmB, &full[s], n0 + lane * 8, k);
-      else if (lane == 16) tma_load_2d(sa, &tmA, &full[s], k, m0);
-    } else if (type == 1) {
-      tma_load_2d(sa + 8 * 1024 + lane * 1024, &tmB, &full[s], n0 + lane * 8, k);
-      if (lane == 0) tma_load_2d(sa, &tmAcs, &full[s], k, m0);
-    } else {
-      if (lane < 8) tma_load_2d(sa + 32 * 1024 + lane * 1024, &tmBcs, &full[s], n0 + lane * 8, k);
-      else if (lane < 10) tma_load_2d(sa + (lane - 8) * 16 * 1024, &tmA, &full[s], k, m0 + (lane - 8) * 128);
-    }
-    __syncwarp();
-    if (lane == 0) {  // advance the cursor
-      if (jn + 1 < njobs) {
-        if (kt + 1 < args.nk && (jn + 1) != args.waves * args.nk) {
-          cur[0] = jn + 1;
-          cur[2] = kt + 1;
-        } else {
-          decode(jn + 1);
-        }
-      }
-    }
-    __syncwarp();
-  };
-  if (warp == 0) {
+  // ---------------- TMA producer warp: streams every job of this CTA through the ring,
+  // refilling a stage as soon as the 4 MMA warps released it (empty mbarrier).  The box
+  // copies are spread over the lanes (one cp.async.bulk.tensor per lane).
+  if (warp == NCW) {
     if (lane == 0) {
       tma_prefetch_desc(&tmA);
       tma_prefetch_desc(&tmB);
       tma_prefetch_desc(&tmAcs);
       tma_prefetch_desc(&tmBcs);
-      if (njobs > 0) decode(0);
     }
-    __syncwarp();
-    for (int jn = 0; jn < STAGES && jn < njobs; ++jn) issue_warp();
+    int tile = -1, kt = 0;
+    Tile tl{0, 0, 0};
+    for (int jn = 0; jn < njobs; ++jn) {
+      if (tile < 0 || kt + 1 >= args.nk || jn == args.waves * args.nk) {
+        iter_of(args, jn, sk0, tile, kt);
+        tl = tile_of(args, tile);
+      } else {
+        ++kt;
+      }
+      const int s = jn % STAGES;
+      if (jn >= STAGES) mbar_wait(&empty[s], (uint32_t)(((jn / STAGES) & 1) ^ 1));
+      uint8_t *sa = smem + s * STAGE_BYTES;
+      const int k = kt * BK;
+      if (lane == 0) mbar_arrive_expect_tx(&full[s], STAGE_BYTES);
+      __syncwarp();
+      if (lane < 8) {
+        tma_load_2d(sa + A_BYTES + lane * 1024, tl.type == 2 ? &tmBcs : &tmB, &full[s],
+                    tl.n0 + lane * 8, k);
+      } else if (lane == 8) {
+        tma_load_2d(sa, tl.type == 1 ? &tmAcs : &tmA, &full[s], k, tl.m0);
+      }
+      __syncwarp();
+    }
+    return;
   }
 
-  double acc[4][4][4];
+  // Fragment addressing.  The mma k index (= tig) of k4-step ks maps to the k-tile column
+  //   k = pi(ks, tig) = (tig&1) | (ks&1)<<1 | ((tig>>1)^(ks>>1))<<2 | (tig>>1)<<3
+  // (a bijection of [0,16); the same permutation for A and B leaves the product unchanged).
+  // With the 128B-swizzled A tile and the 64B-swizzled B boxes every half-warp of a 64-bit
+  // LDS touches 16 distinct 8-byte bank slots (conflict-free: 2 wavefronts).
+  uint32_t offA[4], offB[4];
+#pragma unroll
+  for (int ks = 0; ks < 4; ++ks) {
+    const int k = (tig & 1) | ((ks & 1) << 1) | ((((tig >> 1) ^ (ks >> 1)) & 1) << 2) | ((tig >> 1) << 3);
+    offA[ks] = (uint32_t)(((wm * 32 + g) * 16 + ((((k >> 1) ^ g) << 1) | (k & 1))) * 8);
+    offB[ks] = (uint32_t)(A_BYTES + wn * 4 * 1024 +
+                          (k * 8 + ((((g >> 1) ^ ((k >> 1) & 3)) << 1) | (g & 1))) * 8);
+  }
+
+  double acc[MT][NT][4];
   int j = 0;
   while (j < njobs) {
     // ---------------- segment = consecutive k-tiles of one tile
-    int64_t tile;
-    int kt0;
+    int tile, kt0;
     iter_of(args, j, sk0, tile, kt0);
     const Tile tl = tile_of(args, tile);
-    const int seg_len = (int)(args.nk - kt0 < njobs - j ? args.nk - kt0 : njobs - j);
+    const int seg_len = min(args.nk - kt0, njobs - j);
     const int kt_end = kt0 + seg_len;  // exclusive
-
-    int arow, bbox0, boff;
-    int64_t rbase, cbase;
-    if (tl.type == 0) {
-      arow = wm * 64; bbox0 = wn * 4; boff = 16 * 1024;
-      rbase = tl.m0 + wm * 64; cbase = tl.n0 + wn * 32;
-    } else if (tl.type == 1) {
-      arow = 0; bbox0 = wm * 16 + wn * 4; boff = 8 * 1024;
-      rbase = tl.m0; cbase = tl.n0 + wm * 128 + wn * 32;
-    } else {
-      const int rb = wm + 2 * (wn >> 1);
-      arow = rb * 64; bbox0 = (wn & 1) * 4; boff = 32 * 1024;
-      rbase = tl.m0 + rb * 64; cbase = tl.n0 + (wn & 1) * 32;
-    }
-    // Fragment addressing.  The mma k index (= tig) of k4-step ks maps to the k-tile column
-    //   k = pi(ks, tig) = (tig&1) | (ks&1)<<1 | ((tig>>1)^(ks>>1))<<2 | (tig>>1)<<3
-    // (a bijection of [0,16); the same permutation for A and B leaves the product unchanged).
-    // With the 128B-swizzled A tile and the 64B-swizzled B boxes every half-warp of a 64-bit
-    // LDS touches 16 distinct 8-byte bank slots (conflict-free: 2 wavefronts).
-    uint32_t offA[4], offB[4];
-#pragma unroll
-    for (int ks = 0; ks < 4; ++ks) {
-      const int k = (tig & 1) | ((ks & 1) << 1) | ((((tig >> 1) ^ (ks >> 1)) & 1) << 2) | ((tig >> 1) << 3);
-      offA[ks] = (uint32_t)(((arow + g) * 16 + ((((k >> 1) ^ g) << 1) | (k & 1))) * 8);
-      offB[ks] = (uint32_t)(boff + bbox0 * 1024 +
-                            (k * 8 + ((((g >> 1) ^ ((k >> 1) & 3)) << 1) | (g & 1))) * 8);
-    }
+    const int64_t rbase = (int64_t)tl.m0 + wm * 32, cbase = (int64_t)tl.n0 + wn * 32;
 
     // faults that hit this tile (output coordinates of the tile's product)
     int nf = 0;
     if (args.nfaults > 0) {
-      __syncthreads();
+      mma_sync_bar();
       if (threadIdx.x == 0) *s_nf = 0;
-      __syncthreads();
-      const int64_t rows = tl.type == 0 ? 128 : (tl.type == 1 ? 64 : 256);
-      const int64_t cols = tl.type == 0 ? 128 : (tl.type == 1 ? 256 : 64);
+      mma_sync_bar();
       for (int f = threadIdx.x; f < args.nfaults; f += THREADS) {
         aabft_fault ft = args.faults[f];
         int64_t r = ft.row, c = ft.col;
@@ -269,7 +247,7 @@ __global__ void __launch_bounds__(THREADS, 1)
         else if (r >= args.M && c < args.N) { ftype = 1; r -= args.M; }
         else if (c >= args.N && r < args.M) { ftype = 2; c -= args.N; }
         else ftype = -1;
-        if (ftype == tl.type && r >= tl.m0 && r < tl.m0 + rows && c >= tl.n0 && c < tl.n0 + cols) {
+        if (ftype == tl.type && r >= tl.m0 && r < tl.m0 + TILE && c >= tl.n0 && c < tl.n0 + TILE) {
           const int slot = atomicAdd(s_nf, 1);
           if (slot < MAXF) {
             ft.row = r;
@@ -278,30 +256,30 @@ __global__ void __launch_bounds__(THREADS, 1)
           }
         }
       }
-      __syncthreads();
+      mma_sync_bar();
       nf = min(*s_nf, MAXF);
     }
 
 #pragma unroll
-    for (int i = 0; i < 4; ++i)
+    for (int i = 0; i < MT; ++i)
 #pragma unroll
-      for (int jj = 0; jj < 4; ++jj)
+      for (int jj = 0; jj < NT; ++jj)
 #pragma unroll
         for (int q = 0; q < 4; ++q) acc[i][jj][q] = 0.0;
 
     for (int kt = kt0; kt < kt_end; ++kt, ++j) {
-      const int s = (int)(j % STAGES);
+      const int s = j % STAGES;
       mbar_wait(&full[s], (uint32_t)((j / STAGES) & 1));
       const uint8_t *st = smem + s * STAGE_BYTES;
-      double a[2][4][2], b[2][4];
+      double a[2][MT][2], b[2][NT];
       auto load = [&](int buf, int ks) {
 #pragma unroll
-        for (int mt = 0; mt < 4; ++mt) {
+        for (int mt = 0; mt < MT; ++mt) {
           a[buf][mt][0] = *reinterpret_cast<const double *>(st + offA[ks] + mt * 2048);
           a[buf][mt][1] = *reinterpret_cast<const double *>(st + offA[ks] + mt * 2048 + 1024);
         }
 #pragma unroll
-        for (int nt = 0; nt < 4; ++nt)
+        for (int nt = 0; nt < NT; ++nt)
           b[buf][nt] = *reinterpret_cast<const double *>(st + offB[ks] + nt * 1024);
       };
       load(0, 0);
@@ -309,32 +287,22 @@ __global__ void __launch_bounds__(THREADS, 1)
       for (int ks = 0; ks < BK / 4; ++ks) {
         if (ks + 1 < BK / 4) load((ks + 1) & 1, ks + 1);
 #pragma unroll
-        for (int mt = 0; mt < 4; ++mt)
+        for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
-          for (int nt = 0; nt < 4; ++nt)
+          for (int nt = 0; nt < NT; ++nt)
             dmma(acc[mt][nt], a[ks & 1][mt][0], a[ks & 1][mt][1], b[ks & 1][nt]);
       }
-      // release the stage; the last of the 8 warps refills it with job j + STAGES
+      // release the stage to the producer
       __syncwarp();
-      uint32_t prev = 0;
-      if (lane == 0) {
-        __threadfence_block();
-        prev = atomicAdd(&s_rel[s], 1u);
-      }
-      prev = __shfl_sync(0xffffffffu, prev, 0);
-      if (prev == (uint32_t)(NCW * (j / STAGES + 1) - 1) && j + STAGES < njobs) {
-        __threadfence_block();
-        fence_proxy_async();
-        issue_warp();
-      }
+      if (lane == 0) mbar_arrive(&empty[s]);
       if (nf > 0) {  // Alg 3 errorVecAdd1 at k-tile granularity
         for (int f = 0; f < nf; ++f) {
           const aabft_fault ft = s_f[f];
           if (ft.site != 1 || ft.k_step / BK != kt) continue;
 #pragma unroll
-          for (int mt = 0; mt < 4; ++mt)
+          for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
-            for (int nt = 0; nt < 4; ++nt)
+            for (int nt = 0; nt < NT; ++nt)
 #pragma unroll
               for (int q = 0; q < 4; ++q) {
                 const int64_t r = rbase + mt * 16 + g + (q >> 1) * 8;
@@ -351,37 +319,36 @@ __global__ void __launch_bounds__(THREADS, 1)
       // contributor: park the partial accumulators, then signal the owner
       double *slot = args.partials + (int64_t)blockIdx.x * ACC * THREADS + threadIdx.x;
 #pragma unroll
-      for (int mt = 0; mt < 4; ++mt)
+      for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
-        for (int nt = 0; nt < 4; ++nt)
+        for (int nt = 0; nt < NT; ++nt)
 #pragma unroll
-          for (int q = 0; q < 4; ++q) slot[((mt * 4 + nt) * 4 + q) * THREADS] = acc[mt][nt][q];
+          for (int q = 0; q < 4; ++q) slot[((mt * NT + nt) * 4 + q) * THREADS] = acc[mt][nt][q];
       __threadfence();
-      __syncthreads();
+      mma_sync_bar();
       if (threadIdx.x == 0) atomicExch(&args.flags[blockIdx.x], 1);
       continue;
     }
     if (!last) {
       // owner of a split tile: add the partials of the following CTAs in ascending k order
-      const int64_t tile_it_end = (tile - (int64_t)args.waves * gridDim.x + 1) * args.nk;
+      const int64_t tile_it_end = (int64_t)(tile - args.waves * (int)gridDim.x + 1) * args.nk;
       for (int64_t c = blockIdx.x + 1; c < gridDim.x && sk_begin(args, c) < tile_it_end; ++c) {
         if (sk_begin(args, c + 1) == sk_begin(args, c)) continue;  // empty slice: no partial
         if (threadIdx.x == 0) {
           while (atomicAdd(&args.flags[c], 0) == 0) __nanosleep(64);
           atomicExch(&args.flags[c], 0);  // re-arm for the next launch
           __threadfence();
-          *s_flag = 1;
         }
-        __syncthreads();
+        mma_sync_bar();
         const double *slot = args.partials + c * ACC * THREADS + threadIdx.x;
 #pragma unroll
-        for (int mt = 0; mt < 4; ++mt)
+        for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
-          for (int nt = 0; nt < 4; ++nt)
+          for (int nt = 0; nt < NT; ++nt)
 #pragma unroll
             for (int q = 0; q < 4; ++q)
-              acc[mt][nt][q] += __ldcg(slot + ((mt * 4 + nt) * 4 + q) * THREADS);
-        __syncthreads();
+              acc[mt][nt][q] += __ldcg(slot + ((mt * NT + nt) * 4 + q) * THREADS);
+        mma_sync_bar();
       }
     }
     if (nf > 0) {
@@ -389,9 +356,9 @@ __global__ void __launch_bounds__(THREADS, 1)
         const aabft_fault ft = s_f[f];
         if (ft.site == 1) continue;
 #pragma unroll
-        for (int mt = 0; mt < 4; ++mt)
+        for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
-          for (int nt = 0; nt < 4; ++nt)
+          for (int nt = 0; nt < NT; ++nt)
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
               const int64_t r = rbase + mt * 16 + g + (q >> 1) * 8;
@@ -409,13 +376,13 @@ __global__ void __launch_bounds__(THREADS, 1)
     else { out = args.Crow; ld = args.ld_crow; rows_valid = args.M; cols_valid = args.Ncs; }
     const bool vec_ok = (ld % 2 == 0) && ((reinterpret_cast<uintptr_t>(out) & 15) == 0);
 #pragma unroll
-    for (int mt = 0; mt < 4; ++mt)
+    for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
         const int64_t r = rbase + mt * 16 + g + h * 8;
         if (r >= rows_valid) continue;
 #pragma unroll
-        for (int nt = 0; nt < 4; ++nt) {
+        for (int nt = 0; nt < NT; ++nt) {
           const int64_t c = cbase + nt * 8 + tig * 2;
           double *p = out + r * ld + c;
           const double v0 = acc[mt][nt][h * 2], v1 = acc[mt][nt][h * 2 + 1];
@@ -476,16 +443,20 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
                              int64_t ldb, const aabft_encoded *enc, const aabft_product *out,
                              const aabft_fault *faults, int32_t nfaults, bool plain, void *ws,
                              cudaStream_t st) {
-  static int num_sms = 0;
-  if (!num_sms) {
-    int dev = 0;
+  static int max_ctas = 0;
+  if (!max_ctas) {
+    int dev = 0, sms = 0, per_sm = 0;
     cudaGetDevice(&dev);
-    if (cudaDeviceGetAttribute(&num_sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
       return check_launch("gemm_f64 SM count");
     if (cudaFuncSetAttribute(gemm_f64_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              SMEM_BYTES) != cudaSuccess)
       return check_launch("gemm_f64 smem attribute");
-    num_sms = std::min(num_sms, kMaxCtas);
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, gemm_f64_kernel, CTA_THREADS,
+                                                      SMEM_BYTES) != cudaSuccess || per_sm < 1)
+      return check_launch("gemm_f64 occupancy");
+    // every CTA must be resident (split-tile owners wait on later CTAs)
+    max_ctas = std::min(sms * per_sm, kMaxCtas);
   }
   const int64_t M = cfg->M, N = cfg->N, K = cfg->K, bs = cfg->bs;
   GemmArgs a{};
@@ -497,38 +468,39 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
   a.ld_ccol = plain ? 0 : out->ld_ccol;
   a.Crow = plain ? nullptr : static_cast<double *>(out->Crow);
   a.ld_crow = plain ? 0 : out->ld_crow;
-  a.tm0 = (int)((M + 127) / 128);
-  a.tn0 = (int)((N + 127) / 128);
-  a.tm1 = plain ? 0 : (int)((a.Mcs + 63) / 64);
-  a.tn1 = (int)((N + 255) / 256);
-  a.tm2 = (int)((M + 255) / 256);
-  a.tn2 = plain ? 0 : (int)((a.Ncs + 63) / 64);
-  a.n0 = (int64_t)a.tm0 * a.tn0;
-  a.n1 = (int64_t)a.tm1 * a.tn1;
-  a.n2 = (int64_t)a.tm2 * a.tn2;
-  a.ntiles = a.n0 + a.n1 + a.n2;
-  a.nk = (int)((K + BK - 1) / BK);
-  const int64_t total = a.ntiles * a.nk;
-  const int grid = (int)std::min<int64_t>(num_sms, total);
+  const int64_t tm0 = (M + TILE - 1) / TILE, tn0 = (N + TILE - 1) / TILE;
+  const int64_t tm1 = (a.Mcs + TILE - 1) / TILE, tn2 = (a.Ncs + TILE - 1) / TILE;
+  const int64_t ntiles = tm0 * tn0 + tm1 * tn0 + tm0 * tn2;
+  const int64_t nk = (K + BK - 1) / BK;
+  if (ntiles * nk >= ((int64_t)1 << 31) || M >= ((int64_t)1 << 31) || N >= ((int64_t)1 << 31)) {
+    set_error("gemm_f64: problem too large for 32-bit tile/iteration indices");
+    return AABFT_EINVAL;
+  }
+  a.tm0 = (int)tm0; a.tn0 = (int)tn0; a.tm1 = (int)tm1; a.tn2 = (int)tn2;
+  a.n0 = (int)(tm0 * tn0); a.n1 = (int)(tm1 * tn0); a.n2 = (int)(tm0 * tn2);
+  a.ntiles = (int)ntiles;
+  a.nk = (int)nk;
+  const int64_t total = ntiles * nk;
+  const int grid = (int)std::min<int64_t>(max_ctas, total);
   // full data-parallel waves, keeping at least ~1/2 wave of tiles for the stream-K tail so
   // every CTA's k-slice stays long enough to amortise its fixup
-  int waves = (int)(a.ntiles / grid);
-  if (waves > 0 && a.ntiles % grid != 0 && (a.ntiles % grid) * 2 < grid) waves -= 1;
+  int waves = (int)(ntiles / grid);
+  if (waves > 0 && ntiles % grid != 0 && (ntiles % grid) * 2 < grid) waves -= 1;
   a.waves = waves;
-  a.sk_iters = (a.ntiles - (int64_t)waves * grid) * a.nk;
+  a.sk_iters = (ntiles - (int64_t)waves * grid) * nk;
   a.partials = static_cast<double *>(ws);
   a.flags = reinterpret_cast<int *>(static_cast<char *>(ws) + (size_t)kMaxCtas * ACC * THREADS * sizeof(double));
   a.faults = faults;
   a.nfaults = faults ? nfaults : 0;
 
   CUtensorMap tA, tAcs, tB, tBcs;
-  if (!make_map(&tA, A, K, M, lda, BK, 128, CU_TENSOR_MAP_SWIZZLE_128B)) return AABFT_EINVAL;
+  if (!make_map(&tA, A, K, M, lda, BK, TILE, CU_TENSOR_MAP_SWIZZLE_128B)) return AABFT_EINVAL;
   if (!make_map(&tB, B, N, K, ldb, 8, BK, CU_TENSOR_MAP_SWIZZLE_64B)) return AABFT_EINVAL;
   if (plain) {
     tAcs = tA;
     tBcs = tB;
   } else {
-    if (!make_map(&tAcs, enc->Acs, K, a.Mcs, enc->ld_acs, BK, 64, CU_TENSOR_MAP_SWIZZLE_128B))
+    if (!make_map(&tAcs, enc->Acs, K, a.Mcs, enc->ld_acs, BK, TILE, CU_TENSOR_MAP_SWIZZLE_128B))
       return AABFT_EINVAL;
     if (!make_map(&tBcs, enc->Bcs, a.Ncs, K, enc->ld_bcs, 8, BK, CU_TENSOR_MAP_SWIZZLE_64B))
       return AABFT_EINVAL;
@@ -536,7 +508,7 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
   if (total > 0) {
     if (a.sk_iters > 0 && cudaMemsetAsync(a.flags, 0, kMaxCtas * sizeof(int), st) != cudaSuccess)
       return check_launch("gemm_f64 flag reset");
-    gemm_f64_kernel<<<grid, THREADS, SMEM_BYTES, st>>>(tA, tAcs, tB, tBcs, a);
+    gemm_f64_kernel<<<grid, CTA_THREADS, SMEM_BYTES, st>>>(tA, tAcs, tB, tBcs, a);
     next_launch();
   }
   return check_launch("aabft_gemm(f64)");
