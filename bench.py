@@ -76,10 +76,9 @@ def shard(wl, rank, world):
     if wl["scaling"] == "weak":
         m_local = wl["M"]
         return rank * m_local, m_local, m_local * world
-    M = wl["M"]
-    assert M % (world * wl["bs"]) == 0
-    m_local = M // world
-    return rank * m_local, m_local, M
+    from paper_conf_dsn_braunhw14_b200.distributed import shard_rows
+    row0, m_local = shard_rows(wl["M"], world, rank, wl["bs"])
+    return row0, m_local, wl["M"]
 
 
 # ------------------------------------------------------------------------------- clocks
@@ -231,11 +230,12 @@ def main():
     C_plain = torch.empty(m_local, N, dtype=tdt, device=dev)
     stream = torch.cuda.current_stream(dev)
 
+    from paper_conf_dsn_braunhw14_b200.distributed import reduce_counts
+
     def step():
         plan.run(A, B)
         if world > 1:
-            dist.all_reduce(plan.counts[:8], op=dist.ReduceOp.SUM)
-            dist.all_reduce(plan.counts[8:9].view(torch.float64), op=dist.ReduceOp.MAX)
+            reduce_counts(plan.counts)  # the path's one exchange: SUM counters, MAX ratio
 
     def timed(fn, steps, per_step_events=None):
         if world > 1:

@@ -74,6 +74,32 @@ __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, 
     __syncthreads();
   }
   if (kin) Acs[I * ld_acs + k] = sum;
+  // partial top-p of the checksum row I over this chunk (Alg 1 localSums / maxReduce)
+  {
+    __shared__ double s_v[kEncAChunk / 32][P];
+    __shared__ int s_i[kEncAChunk / 32][P];
+    double v[P];
+    int ix[P];
+    tp_init<P>(v, ix);
+    if (kin) tp_insert<P>(v, ix, fabs((double)sum), (int)k);
+#pragma unroll
+    for (int m = 16; m >= 1; m >>= 1) tp_shfl_merge<P>(v, ix, m);
+    if ((c & 31) == 0) {
+#pragma unroll
+      for (int s = 0; s < P; ++s) { s_v[c >> 5][s] = v[s]; s_i[c >> 5][s] = ix[s]; }
+    }
+    __syncthreads();
+    if (c == 0) {
+      for (int w = 1; w < kEncAChunk / 32; ++w)
+#pragma unroll
+        for (int s = 0; s < P; ++s) tp_insert<P>(v, ix, s_v[w][s], s_i[w][s]);
+      const int64_t row = (int64_t)gridDim.y * bs + I;  // checksum rows follow the M data rows
+      double *dv = pv + (row * nch + chunk) * P;
+      int *di = pi + (row * nch + chunk) * P;
+#pragma unroll
+      for (int s = 0; s < P; ++s) { dv[s] = v[s]; di[s] = ix[s]; }
+    }
+  }
 }
 
 // ---------------------------------------------------------------------------------- B
@@ -92,7 +118,10 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
   const int kc = blockIdx.y;
   const int64_t kbeg = (int64_t)kc * kEncBChunk;
   const int64_t kend = K < kbeg + kEncBChunk ? K : kbeg + kEncBChunk;
-  const int nblk = NC / bs;  // checksum blocks covered by this CTA
+  const int nblk = NC / bs;  // checksum blocks covered by this CTA (<= 16)
+  __shared__ double s_cv[16][P];
+  __shared__ int s_ci[16][P];
+  if (c < 16 * P) { s_cv[c / P][c % P] = -1.0; s_ci[c / P][c % P] = -1; }
   double v[P];
   int ix[P];
   tp_init<P>(v, ix);
@@ -110,17 +139,38 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
       }
     }
     __syncthreads();
-    // Eq 2 row checksums: one thread per (row, block), sequential ascending j
-    for (int task = c; task < SB * nblk; task += NC) {
-      const int rr = task % SB, jb = task / SB;
+    // Eq 2 row checksums: lane rr of the warp owning block jb sums row rr sequentially
+    // (ascending j), then the warp folds the strip's |Bcs| into the running top-p of
+    // checksum column J (partial over this k-chunk)
+    for (int jb = c >> 5; jb < nblk; jb += NC / 32) {
+      const int rr = c & 31;
       const int64_t J = (int64_t)blockIdx.x * nblk + jb;
+      double lv[P];
+      int li[P];
+      tp_init<P>(lv, li);
       if (rr < rows && J * bs < N) {
-        T s = T(0);
-        for (int jj = 0; jj < bs; ++jj) s = s + tile[rr][jb * bs + jj];
-        Bcs[(k0 + rr) * ld_bcs + J] = s;
+        T sm = T(0);
+        for (int jj = 0; jj < bs; ++jj) sm = sm + tile[rr][jb * bs + jj];
+        Bcs[(k0 + rr) * ld_bcs + J] = sm;
+        tp_insert<P>(lv, li, fabs((double)sm), (int)(k0 + rr));
+      }
+#pragma unroll
+      for (int m = 16; m >= 1; m >>= 1) tp_shfl_merge<P>(lv, li, m);
+      if (rr == 0) {
+#pragma unroll
+        for (int r = 0; r < P; ++r) tp_insert<P>(lv, li, s_cv[jb][r], s_ci[jb][r]);
+#pragma unroll
+        for (int r = 0; r < P; ++r) { s_cv[jb][r] = lv[r]; s_ci[jb][r] = li[r]; }
       }
     }
     __syncthreads();
+  }
+  if (c < nblk && ((int64_t)blockIdx.x * nblk + c) * bs < N) {
+    const int64_t J = (int64_t)blockIdx.x * nblk + c;
+    double *dv = pv + ((N + J) * nch + kc) * P;
+    int *di = pi + ((N + J) * nch + kc) * P;
+#pragma unroll
+    for (int r = 0; r < P; ++r) { dv[r] = s_cv[c][r]; di[r] = s_ci[c][r]; }
   }
   if (jin) {
     double *dv = pv + (j * nch + kc) * P;
@@ -131,8 +181,8 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
 }
 
 // ---------------------------------------------------------------------------------- step 3
-// One warp per vector: data rows of A / data cols of B merge their per-chunk partial lists;
-// checksum rows of Acs / checksum cols of Bcs are scanned directly.
+// One warp per vector (data rows + checksum rows of A, data cols + checksum cols of B): merge
+// the per-chunk partial lists produced by the encode kernels.
 template <typename T, int P>
 __global__ void __launch_bounds__(256) topp_reduce_kernel(
     int64_t M, int64_t N, int64_t K, int bs, const double *__restrict__ pva,
@@ -152,27 +202,16 @@ __global__ void __launch_bounds__(256) topp_reduce_kernel(
   double *ov;
   int *oi;
   if (w < nA) {
-    if (w < M) {
-      const double *sv = pva + w * ncha * P;
-      const int *si = pia + w * ncha * P;
-      for (int e = lane; e < ncha * P; e += 32) tp_insert<P>(v, ix, sv[e], si[e]);
-    } else {
-      const T *row = Acs + (w - M) * ld_acs;
-      for (int64_t k = lane; k < K; k += 32) tp_insert<P>(v, ix, fabs((double)row[k]), (int)k);
-    }
+    const double *sv = pva + w * ncha * P;
+    const int *si = pia + w * ncha * P;
+    for (int e = lane; e < ncha * P; e += 32) tp_insert<P>(v, ix, sv[e], si[e]);
     ov = topA_v + w * P;
     oi = topA_i + w * P;
   } else {
     const int64_t u = w - nA;
-    if (u < N) {
-      const double *sv = pvb + u * nchb * P;
-      const int *si = pib + u * nchb * P;
-      for (int e = lane; e < nchb * P; e += 32) tp_insert<P>(v, ix, sv[e], si[e]);
-    } else {
-      const T *col = Bcs + (u - N);
-      for (int64_t k = lane; k < K; k += 32)
-        tp_insert<P>(v, ix, fabs((double)col[k * ld_bcs]), (int)k);
-    }
+    const double *sv = pvb + u * nchb * P;
+    const int *si = pib + u * nchb * P;
+    for (int e = lane; e < nchb * P; e += 32) tp_insert<P>(v, ix, sv[e], si[e]);
     ov = topB_v + u * P;
     oi = topB_i + u * P;
   }
@@ -191,12 +230,13 @@ aabft_status run_encode(const aabft_config *cfg, const T *A, int64_t lda, const 
   const int bs = cfg->bs;
   const int ncha = (int)enc_a_chunks(K), nchb = (int)enc_b_chunks(K);
   char *w = static_cast<char *>(ws);
+  const size_t ra = (size_t)(M + M / bs), rb = (size_t)(N + N / bs);
   double *pva = reinterpret_cast<double *>(w);
-  w += ((size_t)M * ncha * P * 8 + 255) / 256 * 256;
+  w += (ra * ncha * P * 8 + 255) / 256 * 256;
   int *pia = reinterpret_cast<int *>(w);
-  w += ((size_t)M * ncha * P * 4 + 255) / 256 * 256;
+  w += (ra * ncha * P * 4 + 255) / 256 * 256;
   double *pvb = reinterpret_cast<double *>(w);
-  w += ((size_t)N * nchb * P * 8 + 255) / 256 * 256;
+  w += (rb * nchb * P * 8 + 255) / 256 * 256;
   int *pib = reinterpret_cast<int *>(w);
   if (A) {
     dim3 grid(ncha, (unsigned)(M / bs));
@@ -249,8 +289,8 @@ size_t encode_ws_bytes(const aabft_config *cfg) {
   const size_t p = (size_t)cfg->p;
   const size_t ncha = (size_t)enc_a_chunks(cfg->K), nchb = (size_t)enc_b_chunks(cfg->K);
   auto r = [](size_t b) { return (b + 255) / 256 * 256; };
-  return r(cfg->M * ncha * p * 8) + r(cfg->M * ncha * p * 4) + r(cfg->N * nchb * p * 8) +
-         r(cfg->N * nchb * p * 4);
+  const size_t ra = (size_t)(cfg->M + cfg->M / cfg->bs), rb = (size_t)(cfg->N + cfg->N / cfg->bs);
+  return r(ra * ncha * p * 8) + r(ra * ncha * p * 4) + r(rb * nchb * p * 8) + r(rb * nchb * p * 4);
 }
 
 aabft_status launch_encode(const aabft_config *cfg, const void *A, int64_t lda, const void *B,

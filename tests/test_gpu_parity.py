@@ -365,3 +365,24 @@ def test_full_size_c2_sampled(P, orc):
         assert np.array_equal(tbv[N + J], ob["enc"]["topB"][0][bs])
         assert ob["check"].status[0, 0] == res.reports()["status"][I, J] == 0
         assert norm_err(C[I * bs:(I + 1) * bs, J * bs:(J + 1) * bs], ob["C"], Ab, Bb) <= 1e-13
+
+
+def test_distributed_single_rank_nccl(P, orc):
+    """The distributed driver (row shard + NCCL counter all-reduce) at world size 1."""
+    import os
+    import torch.distributed as dist
+    from paper_conf_dsn_braunhw14_b200 import distributed as D
+    if not dist.is_initialized():
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29533")
+        dist.init_process_group("nccl", rank=0, world_size=1)
+    M, N, K, bs = 256, 256, 128, 64
+    A = gen("uniform", M, K, 21, 0)
+    B = gen("uniform", K, N, 21, 1)
+    r0, n = D.shard_rows(M, 1, 0, bs)
+    res, cnt = D.protected_matmul(to_dev(A[r0:r0 + n]), to_dev(B), bs=bs,
+                                  faults=[dict(row=3, col=5, site=2, add=1.0)])
+    torch.cuda.synchronize()
+    assert cnt["blocks"] == 16 and cnt["corrected"] == 1 and cnt["clean"] == 15
+    assert norm_err(host(res.C), orc.gemm(A, B), A, B) <= 1e-13
+    dist.destroy_process_group()
