@@ -92,7 +92,11 @@ typedef struct {
 /* Output of aabft_gemm.  C: M x N (ldc >= N); Ccol: (M/bs) x N (ld_ccol >= N) carried column
  * checksums c_{m+1,j} per block-row; Crow: M x (N/bs) (ld_crow >= N/bs) carried row
  * checksums c_{i,q+1} per block-column (Eq 3 with partitioned encoding; corner not formed,
- * reading R17). */
+ * reading R17).
+ * Rcol / Rrow (optional, double, dense (M/bs) x N and M x (N/bs)): when both are non-NULL and
+ * the FP64 path runs with bs <= 64, aabft_gemm also writes the REFERENCE checksums of Eq 4
+ * (c*_{m+1,j}, c*_{i,q+1}) from its epilogue registers and aabft_check compares those instead
+ * of re-reading C ("fused check").  NULL = unfused: aabft_check re-sums C. */
 typedef struct {
   void *C;
   int64_t ldc;
@@ -100,6 +104,8 @@ typedef struct {
   int64_t ld_ccol;
   void *Crow;
   int64_t ld_crow;
+  double *Rcol;
+  double *Rrow;
 } aabft_product;
 
 /* Per-block (BS x BS sub-matrix of C, "one threadblock for each submatrix of C")
@@ -137,7 +143,10 @@ typedef struct {
  *  site 1: XOR xor_mask into the accumulator after the k-tile that contains k_step
  *          ("errorVecAdd1" at k-tile granularity; products inside the DMMA unit
  *          are not addressable)
- *  site 2: add `add` to the stored result (magnitude sweep) */
+ *  site 2: add `add` to the stored result (magnitude sweep)
+ * Capacity: the FP64 kernel applies at most 64 faults per 64 x 64 tile of C / Ccol / Crow, the
+ * FP32 kernel at most 256 per 128 x 128 tile (i.e. one per 8 x 8 block); extra faults in the
+ * same tile are ignored. */
 typedef struct {
   int64_t row, col;
   int32_t site;

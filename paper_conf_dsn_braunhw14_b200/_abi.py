@@ -39,7 +39,8 @@ class Encoded(C.Structure):
 
 class Product(C.Structure):
     _fields_ = [("C", C.c_void_p), ("ldc", C.c_int64), ("Ccol", C.c_void_p),
-                ("ld_ccol", C.c_int64), ("Crow", C.c_void_p), ("ld_crow", C.c_int64)]
+                ("ld_ccol", C.c_int64), ("Crow", C.c_void_p), ("ld_crow", C.c_int64),
+                ("Rcol", C.c_void_p), ("Rrow", C.c_void_p)]
 
 
 class BlockReport(C.Structure):

@@ -98,7 +98,8 @@ class ProtectedGemm:
     """Pre-allocated buffers + ABI structs for repeated protected GEMMs of one shape."""
 
     def __init__(self, M: int, N: int, K: int, *, dtype=torch.float64, bs: int = 64, p: int = 2,
-                 omega: float = 3.0, t: int = 0, fma_model: int = 1, device=None):
+                 omega: float = 3.0, t: int = 0, fma_model: int = 1, device=None,
+                 fused: bool = True):
         lib()  # fail loudly before allocating anything
         self.device = torch.device("cuda" if device is None else device)
         self.dtype = dtype
@@ -130,8 +131,12 @@ class ProtectedGemm:
         self.enc = Encoded(self._Acs.data_ptr(), self.ld_acs, self._Bcs.data_ptr(), self.ld_bcs,
                            self.topA_val.data_ptr(), self.topA_idx.data_ptr(),
                            self.topB_val.data_ptr(), self.topB_idx.data_ptr())
+        # fused check (FP64, bs <= 64): the GEMM epilogue writes the reference sums
+        self.fused = bool(fused and dtype == torch.float64 and bs <= 64)
+        self.Rcol = torch.empty(nI, N, dtype=torch.float64, device=dev) if self.fused else None
+        self.Rrow = torch.empty(M, nJ, dtype=torch.float64, device=dev) if self.fused else None
         self.prod = Product(self._C.data_ptr(), self.ldc, self._Ccol.data_ptr(), self.ld_ccol,
-                            self._Crow.data_ptr(), self.ld_crow)
+                            self._Crow.data_ptr(), self.ld_crow, _ptr(self.Rcol), _ptr(self.Rrow))
 
     # views without the pitch padding
     @property

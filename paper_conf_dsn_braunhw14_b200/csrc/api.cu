@@ -262,7 +262,7 @@ aabft_status aabft_correct(const aabft_config *cfg, const aabft_encoded *enc,
 namespace {
 struct Arena {
   int64_t lda, ldb, ldc, ld_acs, ld_bcs, ld_ccol, ld_crow;
-  size_t oA, oB, oC, oAcs, oBcs, oCcol, oCrow, oTav, oTai, oTbv, oTbi, oRep, oCnt, oWs, total;
+  size_t oA, oB, oC, oAcs, oBcs, oCcol, oCrow, oRcol, oRrow, oTav, oTai, oTbv, oTbi, oRep, oCnt, oWs, total;
 };
 Arena plan_arena(const aabft_config *c) {
   Arena a;
@@ -281,6 +281,8 @@ Arena plan_arena(const aabft_config *c) {
   a.oBcs = take(c->K * a.ld_bcs * es);
   a.oCcol = take((c->M / c->bs) * a.ld_ccol * es);
   a.oCrow = take(c->M * a.ld_crow * es);
+  a.oRcol = take((c->M / c->bs) * c->N * 8);
+  a.oRrow = take(c->M * (c->N / c->bs) * 8);
   a.oTav = take((c->M + c->M / c->bs) * c->p * 8);
   a.oTai = take((c->M + c->M / c->bs) * c->p * 4);
   a.oTbv = take((c->N + c->N / c->bs) * c->p * 8);
@@ -318,7 +320,8 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
   aabft_encoded enc{base + a.oAcs, a.ld_acs, base + a.oBcs, a.ld_bcs,
                     reinterpret_cast<double *>(base + a.oTav), reinterpret_cast<int32_t *>(base + a.oTai),
                     reinterpret_cast<double *>(base + a.oTbv), reinterpret_cast<int32_t *>(base + a.oTbi)};
-  aabft_product prod{base + a.oC, a.ldc, base + a.oCcol, a.ld_ccol, base + a.oCrow, a.ld_crow};
+  aabft_product prod{base + a.oC, a.ldc, base + a.oCcol, a.ld_ccol, base + a.oCrow, a.ld_crow,
+                     reinterpret_cast<double *>(base + a.oRcol), reinterpret_cast<double *>(base + a.oRrow)};
   auto *rep = reinterpret_cast<aabft_block_report *>(base + a.oRep);
   auto *cnt = reinterpret_cast<aabft_counts *>(base + a.oCnt);
   const size_t wsb = aabft_workspace_bytes(cfg);

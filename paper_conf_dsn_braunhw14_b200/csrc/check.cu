@@ -118,7 +118,39 @@ struct CheckArgs {
   const int *tbi;
   aabft_block_report *rep;
   aabft_counts *cnt;
+  const double *Rcol;  // fused reference sums from the GEMM epilogue (NULL = re-sum C)
+  const double *Rrow;
 };
+
+// block verdict + report + aggregated counter update (shared by both check kernels)
+__device__ __forceinline__ void finish_block(const CheckArgs &a, int64_t blk, int nr, int nc,
+                                             int crit_row, int crit_col, const int cls[3],
+                                             double br) {
+  uint8_t status;
+  if (nr == 0 && nc == 0) status = AABFT_BLK_CLEAN;
+  else if (nr == 1 && nc == 1) status = AABFT_BLK_SINGLE;
+  else if (nr == 0 || nc == 0) status = AABFT_BLK_CHECKSUM_ONLY;
+  else status = AABFT_BLK_UNCORRECTABLE;
+  aabft_block_report r;
+  r.status = status;
+  r.worst_class = (uint8_t)(cls[2] ? 2 : (cls[1] ? 1 : 0));
+  r.n_bad_rows = (uint16_t)min(nr, 65535);
+  r.n_bad_cols = (uint16_t)min(nc, 65535);
+  r.reserved = 0;
+  r.row = status == AABFT_BLK_SINGLE ? crit_row : -1;
+  r.col = status == AABFT_BLK_SINGLE ? crit_col : -1;
+  r.max_ratio = (float)br;
+  a.rep[blk] = r;
+  unsigned long long *n = reinterpret_cast<unsigned long long *>(a.cnt->n);
+  atomicAdd(&n[0], 1ull);
+  if (status == AABFT_BLK_CLEAN) atomicAdd(&n[1], 1ull);
+  if (status == AABFT_BLK_CHECKSUM_ONLY) atomicAdd(&n[3], 1ull);
+  if (status == AABFT_BLK_UNCORRECTABLE) atomicAdd(&n[4], 1ull);
+  for (int c = 0; c < 3; ++c)
+    if (cls[c]) atomicAdd(&n[5 + c], (unsigned long long)cls[c]);
+  if (br > 0.0) atomicMax(reinterpret_cast<unsigned long long *>(&a.cnt->max_ratio),
+                          (unsigned long long)__double_as_longlong(br));
+}
 
 template <typename T, int P>
 __global__ void __launch_bounds__(kCheckThreads) check_kernel(CheckArgs a, BoundParams bp) {
@@ -190,30 +222,63 @@ __global__ void __launch_bounds__(kCheckThreads) check_kernel(CheckArgs a, Bound
   if (tid == 0) {
     double br = 0.0;
     for (int w = 0; w < kCheckThreads / 32; ++w) br = fmax(br, s_ratio[w]);
-    const int nr = s_nr, nc = s_nc;
-    uint8_t status;
-    if (nr == 0 && nc == 0) status = AABFT_BLK_CLEAN;
-    else if (nr == 1 && nc == 1) status = AABFT_BLK_SINGLE;
-    else if (nr == 0 || nc == 0) status = AABFT_BLK_CHECKSUM_ONLY;
-    else status = AABFT_BLK_UNCORRECTABLE;
-    aabft_block_report r;
-    r.status = status;
-    r.worst_class = (uint8_t)(s_cls[2] ? 2 : (s_cls[1] ? 1 : 0));
-    r.n_bad_rows = (uint16_t)min(nr, 65535);
-    r.n_bad_cols = (uint16_t)min(nc, 65535);
-    r.reserved = 0;
-    r.row = status == AABFT_BLK_SINGLE ? s_row : -1;
-    r.col = status == AABFT_BLK_SINGLE ? s_col : -1;
-    r.max_ratio = (float)br;
-    a.rep[blockIdx.x] = r;
-    unsigned long long *n = reinterpret_cast<unsigned long long *>(a.cnt->n);
-    atomicAdd(&n[0], 1ull);
-    if (status == AABFT_BLK_CLEAN) atomicAdd(&n[1], 1ull);
-    if (status == AABFT_BLK_CHECKSUM_ONLY) atomicAdd(&n[3], 1ull);
-    if (status == AABFT_BLK_UNCORRECTABLE) atomicAdd(&n[4], 1ull);
-    for (int c = 0; c < 3; ++c)
-      if (s_cls[c]) atomicAdd(&n[5 + c], (unsigned long long)s_cls[c]);
-    if (br > 0.0) atomic_max_nonneg(&a.cnt->max_ratio, br);
+    const int cls[3] = {s_cls[0], s_cls[1], s_cls[2]};
+    finish_block(a, blockIdx.x, s_nr, s_nc, s_row, s_col, cls, br);
+  }
+}
+
+// --------------------------------------------------------------------------- fused check
+// The GEMM epilogue already produced the reference sums (Rcol, Rrow); compare them with the
+// carried checksums: 2*bs checks per block, no pass over C.
+template <typename T, int P>
+__global__ void __launch_bounds__(128) check_fused_kernel(CheckArgs a, BoundParams bp) {
+  __shared__ int s_cls[3], s_nr, s_nc, s_row, s_col;
+  __shared__ double s_ratio[4];
+  const int bs = a.bs, tid = threadIdx.x, lane = tid & 31;
+  const int64_t nJ = a.N / bs;
+  const int64_t I = blockIdx.x / nJ, J = blockIdx.x % nJ;
+  if (tid < 3) s_cls[tid] = 0;
+  if (tid == 0) { s_nr = 0; s_nc = 0; s_row = -1; s_col = -1; }
+  __syncthreads();
+  int cls_local[3] = {0, 0, 0};
+  double rmax = 0.0;
+  for (int e = tid; e < 2 * bs; e += 128) {
+    double d;
+    Bound b;
+    if (e < bs) {  // column check j
+      const int64_t j = J * bs + e;
+      d = a.Rcol[I * a.N + j] - (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
+      b = bound_of(bp, y_bound<P>(a.tav + (a.M + I) * P, a.tai + (a.M + I) * P, a.tbv + j * P,
+                                  a.tbi + j * P));
+      const int cl = classify(d, b);
+      cls_local[cl] += 1;
+      if (cl == 2) { atomicAdd(&s_nc, 1); s_col = (int)j; }
+    } else {  // row check i
+      const int64_t i = I * bs + (e - bs);
+      d = a.Rrow[i * nJ + J] - (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
+      b = bound_of(bp, y_bound<P>(a.tav + i * P, a.tai + i * P, a.tbv + (a.N + J) * P,
+                                  a.tbi + (a.N + J) * P));
+      const int cl = classify(d, b);
+      cls_local[cl] += 1;
+      if (cl == 2) { atomicAdd(&s_nr, 1); s_row = (int)i; }
+    }
+    rmax = fmax(rmax, ratio_of(d, b.eps));
+  }
+#pragma unroll
+  for (int c = 0; c < 3; ++c) {
+    int v = cls_local[c];
+#pragma unroll
+    for (int m = 16; m >= 1; m >>= 1) v += __shfl_xor_sync(0xffffffffu, v, m);
+    if (lane == 0 && v) atomicAdd(&s_cls[c], v);
+  }
+#pragma unroll
+  for (int m = 16; m >= 1; m >>= 1) rmax = fmax(rmax, __shfl_xor_sync(0xffffffffu, rmax, m));
+  if (lane == 0) s_ratio[tid >> 5] = rmax;
+  __syncthreads();
+  if (tid == 0) {
+    const double br = fmax(fmax(s_ratio[0], s_ratio[1]), fmax(s_ratio[2], s_ratio[3]));
+    const int cls[3] = {s_cls[0], s_cls[1], s_cls[2]};
+    finish_block(a, blockIdx.x, s_nr, s_nc, s_row, s_col, cls, br);
   }
 }
 
@@ -260,6 +325,10 @@ CheckArgs make_args(const aabft_config *cfg, const aabft_encoded *enc, const aab
   a.tav = enc->topA_val; a.tai = enc->topA_idx;
   a.tbv = enc->topB_val; a.tbi = enc->topB_idx;
   a.rep = rep; a.cnt = cnt;
+  // fused reference sums exist only where aabft_gemm produces them (FP64, bs <= 64)
+  const bool fused = prod->Rcol && prod->Rrow && cfg->dtype == AABFT_F64 && cfg->bs <= 64;
+  a.Rcol = fused ? prod->Rcol : nullptr;
+  a.Rrow = fused ? prod->Rrow : nullptr;
   return a;
 }
 
@@ -273,7 +342,11 @@ aabft_status run_check(const aabft_config *cfg, const CheckArgs &a, BoundParams 
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   }
   if (nb > 0) {
-    kern<<<(unsigned)nb, kCheckThreads, smem, st>>>(a, bp);
+    if (a.Rcol && a.Rrow) {
+      check_fused_kernel<T, P><<<(unsigned)nb, 128, 0, st>>>(a, bp);
+    } else {
+      kern<<<(unsigned)nb, kCheckThreads, smem, st>>>(a, bp);
+    }
     next_launch();
   }
   return check_launch("aabft_check");

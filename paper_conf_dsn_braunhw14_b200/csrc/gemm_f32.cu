@@ -15,7 +15,7 @@ namespace aabft {
 namespace {
 
 constexpr int BM = 128, BN = 128, BK = 8, THREADS = 256, AST = BM + 4;
-constexpr int MAXF = 16;
+constexpr int MAXF = 256;  // faults per 128x128 tile kept in smem (one per 8x8 block)
 constexpr int GROUP_M = 8;
 
 struct SgemmArgs {

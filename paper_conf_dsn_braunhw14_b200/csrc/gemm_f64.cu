@@ -49,10 +49,11 @@ constexpr int MT = 2, NT = 4;               // m16 x n8 fragments per warp: 32 x
 constexpr int A_BYTES = TILE * BK * 8;      // 8 KiB
 constexpr int B_BYTES = BK * TILE * 8;      // 8 KiB
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-constexpr int MAXF = 16;                    // faults per tile kept in smem
+constexpr int MAXF = 64;                    // faults per 64x64 tile kept in smem (one per 8x8 block)
 constexpr int BOOK = 128;                   // barriers, counters, cursor
+constexpr int RED_BYTES = 2 * 2 * 32 * 8;  // cross-warp partial reference sums (BS = 64)
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + BOOK +
-                           MAXF * (int)sizeof(aabft_fault);
+                           MAXF * (int)sizeof(aabft_fault) + RED_BYTES;
 constexpr int GROUP_M = AABFT_F64_GROUP_M;
 constexpr int kMaxCtas = 1024;              // >= resident CTAs; sizes the split-K partial slots
 constexpr int ACC = MT * NT * 4;            // accumulators per thread
@@ -74,6 +75,9 @@ struct GemmArgs {
   int *flags;                         // [kMaxCtas]
   const aabft_fault *faults;
   int nfaults;
+  double *Rcol;                       // fused reference sums (NULL = unfused): (M/bs) x N
+  double *Rrow;                       //                                         M x (N/bs)
+  int bs;
 };
 
 struct Tile {
@@ -154,6 +158,8 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
   int *s_nf = reinterpret_cast<int *>(empty + STAGES);
   static_assert(16 * STAGES + 8 <= BOOK, "bookkeeping fits");
   aabft_fault *s_f = reinterpret_cast<aabft_fault *>(smem + STAGES * STAGE_BYTES + BOOK);
+  double *s_red = reinterpret_cast<double *>(smem + STAGES * STAGE_BYTES + BOOK +
+                                             MAXF * sizeof(aabft_fault));  // [2][2][32]
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int g = lane >> 2, tig = lane & 3;
@@ -369,6 +375,122 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
             }
       }
     }
+    if (args.Rcol != nullptr && tl.type == 0) {
+      // ---- fused reference sums (Eq 4) of the BS x BS blocks inside this 64 x 64 C tile, taken
+      // from the registers that are about to be stored (after any injected fault), in a fixed
+      // order: 8-row/8-column shuffle trees, then pairwise over fragments, then across warps.
+      const int bs = args.bs;
+      const int64_t nJ = args.N / bs;
+      double csum[NT][2], rsum[MT][2];  // per-warp totals (used for BS = 64)
+      // column sums: per (nt, e) column, 8-row shuffle trees then pairwise over (mt, h)
+#pragma unroll
+      for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          double c8[MT][2];
+#pragma unroll
+          for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              double v = acc[mt][nt][h * 2 + e];
+              v += __shfl_xor_sync(0xffffffffu, v, 4);
+              v += __shfl_xor_sync(0xffffffffu, v, 8);
+              v += __shfl_xor_sync(0xffffffffu, v, 16);
+              c8[mt][h] = v;  // rows mt*16 + h*8 + (0..7)
+            }
+          const double c16a = c8[0][0] + c8[0][1], c16b = c8[1][0] + c8[1][1];
+          csum[nt][e] = c16a + c16b;
+          const int64_t col = cbase + nt * 8 + tig * 2 + e;
+          if (bs <= 32 && g == 0 && col < args.N) {
+            if (bs == 8) {
+#pragma unroll
+              for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                  const int64_t I = (rbase + mt * 16 + h * 8) / 8;
+                  if (I * 8 < args.M) args.Rcol[I * args.N + col] = c8[mt][h];
+                }
+            } else if (bs == 16) {
+              const int64_t I0 = rbase / 16;
+              if (I0 * 16 < args.M) args.Rcol[I0 * args.N + col] = c16a;
+              if ((I0 + 1) * 16 < args.M) args.Rcol[(I0 + 1) * args.N + col] = c16b;
+            } else {
+              const int64_t I = rbase / 32;
+              if (I * 32 < args.M) args.Rcol[I * args.N + col] = csum[nt][e];
+            }
+          }
+        }
+      // row sums: per (mt, h) row, pairwise over e, 4-lane shuffle tree, then over nt
+#pragma unroll
+      for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          double r8[NT];
+#pragma unroll
+          for (int nt = 0; nt < NT; ++nt) {
+            double v = acc[mt][nt][h * 2] + acc[mt][nt][h * 2 + 1];
+            v += __shfl_xor_sync(0xffffffffu, v, 1);
+            v += __shfl_xor_sync(0xffffffffu, v, 2);
+            r8[nt] = v;  // columns nt*8 + (0..7)
+          }
+          const double r16a = r8[0] + r8[1], r16b = r8[2] + r8[3];
+          rsum[mt][h] = r16a + r16b;
+          const int64_t row = rbase + mt * 16 + h * 8 + g;
+          if (bs <= 32 && tig == 0 && row < args.M) {
+            if (bs == 8) {
+#pragma unroll
+              for (int nt = 0; nt < NT; ++nt) {
+                const int64_t J = (cbase + nt * 8) / 8;
+                if (J < nJ) args.Rrow[row * nJ + J] = r8[nt];
+              }
+            } else if (bs == 16) {
+              const int64_t J0 = cbase / 16;
+              if (J0 < nJ) args.Rrow[row * nJ + J0] = r16a;
+              if (J0 + 1 < nJ) args.Rrow[row * nJ + J0 + 1] = r16b;
+            } else {
+              const int64_t J = cbase / 32;
+              if (J < nJ) args.Rrow[row * nJ + J] = rsum[mt][h];
+            }
+          }
+        }
+      if (bs == 64) {  // the whole tile is one block: combine the 2 x 2 warps via smem
+        double *s_col = s_red;       // [wn][32]: column partials of the wm = 1 warps
+        double *s_row = s_red + 64;  // [wm][32]: row partials of the wn = 1 warps
+        mma_sync_bar();
+        if (wm == 1 && g == 0) {
+#pragma unroll
+          for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+            for (int e = 0; e < 2; ++e) s_col[wn * 32 + nt * 8 + tig * 2 + e] = csum[nt][e];
+        }
+        if (wn == 1 && tig == 0) {
+#pragma unroll
+          for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) s_row[wm * 32 + mt * 16 + h * 8 + g] = rsum[mt][h];
+        }
+        mma_sync_bar();
+        const int64_t I = (int64_t)tl.m0 / 64, J = (int64_t)tl.n0 / 64;
+        if (wm == 0 && g == 0) {
+#pragma unroll
+          for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+              const int c = wn * 32 + nt * 8 + tig * 2 + e;
+              if (tl.n0 + c < args.N) args.Rcol[I * args.N + tl.n0 + c] = csum[nt][e] + s_col[c];
+            }
+        }
+        if (wn == 0 && tig == 0) {
+#pragma unroll
+          for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              const int r = wm * 32 + mt * 16 + h * 8 + g;
+              if (tl.m0 + r < args.M) args.Rrow[((int64_t)tl.m0 + r) * nJ + J] = rsum[mt][h] + s_row[r];
+            }
+        }
+      }
+    }
     double *out;
     int64_t ld, rows_valid, cols_valid;
     if (tl.type == 0) { out = args.C; ld = args.ldc; rows_valid = args.M; cols_valid = args.N; }
@@ -492,6 +614,10 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
   a.flags = reinterpret_cast<int *>(static_cast<char *>(ws) + (size_t)kMaxCtas * ACC * THREADS * sizeof(double));
   a.faults = faults;
   a.nfaults = faults ? nfaults : 0;
+  a.bs = (int)bs;
+  const bool fused = !plain && out->Rcol && out->Rrow && bs <= TILE;
+  a.Rcol = fused ? out->Rcol : nullptr;
+  a.Rrow = fused ? out->Rrow : nullptr;
 
   CUtensorMap tA, tAcs, tB, tBcs;
   if (!make_map(&tA, A, K, M, lda, BK, TILE, CU_TENSOR_MAP_SWIZZLE_128B)) return AABFT_EINVAL;

@@ -45,7 +45,8 @@ def test_struct_layout_matches_header(tmp_path):
                                              "fma_model"]),
               "aabft_encoded": (_abi.Encoded, ["Acs", "ld_acs", "Bcs", "ld_bcs", "topA_val",
                                                "topA_idx", "topB_val", "topB_idx"]),
-              "aabft_product": (_abi.Product, ["C", "ldc", "Ccol", "ld_ccol", "Crow", "ld_crow"]),
+              "aabft_product": (_abi.Product, ["C", "ldc", "Ccol", "ld_ccol", "Crow", "ld_crow",
+                                               "Rcol", "Rrow"]),
               "aabft_block_report": (_abi.BlockReport, ["status", "worst_class", "n_bad_rows",
                                                         "n_bad_cols", "row", "col", "max_ratio"]),
               "aabft_counts": (_abi.Counts, ["n", "max_ratio"]),
@@ -105,7 +106,7 @@ def test_workspace_and_null_checks(L):
     # workspace too small
     assert L.aabft_encode(C.byref(cfg), 16, 256, None, 0, C.byref(enc), 16, 8, None) == 4
     # misaligned operand for the TMA GEMM
-    prod = _abi.Product(16, 256, 16, 256, 16, 4)
+    prod = _abi.Product(16, 256, 16, 256, 16, 4, None, None)
     st = L.aabft_gemm(C.byref(cfg), 8, 256, 16, 256, C.byref(enc), C.byref(prod), None, 0, 16,
                       1 << 40, None)
     assert st == 1 and b"aligned" in L.aabft_last_error()

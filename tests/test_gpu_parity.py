@@ -59,10 +59,10 @@ def xor_val(v, mask, dtype):
 
 
 def run_both(P, orc, M, N, K, bs, p, dtype=np.float64, recipe="uniform", faults=(), seed=1,
-             correct=True, q=8):
+             correct=True, q=8, fused=True):
     A = gen(recipe, M, K, seed, 0, dtype, q=q)
     B = gen(recipe, K, N, seed, 1, dtype, q=q)
-    plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p)
+    plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p, fused=fused)
     res = plan.run(to_dev(A), to_dev(B), faults=list(faults), correct=correct)
     torch.cuda.synchronize()
     o = orc.protected_matmul(A, B, bs=bs, p=p, faults=list(faults), do_correct=correct)
@@ -167,12 +167,13 @@ def test_gemm_plain_same_family(P, orc):
         assert norm_err(host(Cp), orc.gemm(A, B), A, B) <= (1e-13 if dtype == np.float64 else 1e-5)
 
 
+@pytest.mark.parametrize("fused", [True, False])
 @pytest.mark.parametrize("dtype,recipe", [(np.float64, "uniform"), (np.float64, "positive"),
                                           (np.float64, "wide"), (np.float32, "uniform"),
                                           (np.float32, "wide"), (np.float64, "integer")])
-def test_clean_run_verdicts(P, orc, dtype, recipe):
+def test_clean_run_verdicts(P, orc, dtype, recipe, fused):
     M, N, K, bs, p = 256, 192, 512, 64, 2
-    A, B, plan, res, o = run_both(P, orc, M, N, K, bs, p, dtype=dtype, recipe=recipe)
+    A, B, plan, res, o = run_both(P, orc, M, N, K, bs, p, dtype=dtype, recipe=recipe, fused=fused)
     rep = res.reports()
     cnt = res.counts()
     assert cnt["checks_critical"] == 0 and o["check"].counts[7] == 0
@@ -220,14 +221,17 @@ def _fault_set(orc, A, B, bs, p, rng, dtype, n_per_mag=1):
     return faults, labels
 
 
-@pytest.mark.parametrize("dtype", [np.float64, np.float32])
-def test_fault_verdicts_outside_band(P, orc, dtype):
-    M, N, K, bs, p = 512, 512, 256, 64, 2
+@pytest.mark.parametrize("dtype,fused,bs", [(np.float64, True, 64), (np.float64, False, 64),
+                                            (np.float64, True, 32), (np.float64, True, 16),
+                                            (np.float64, True, 8), (np.float32, False, 64)])
+def test_fault_verdicts_outside_band(P, orc, dtype, fused, bs):
+    M, N, K, p = 512, 512, 256, 2
     rng = np.random.default_rng(42)
     A = gen("uniform", M, K, 11, 0, dtype)
     B = gen("uniform", K, N, 11, 1, dtype)
     faults, labels = _fault_set(orc, A, B, bs, p, rng, dtype)
-    plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p)
+    plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p, fused=fused)
+    assert plan.fused == (fused and dtype == np.float64)
     dA, dB = to_dev(A), to_dev(B)
     clean = host(plan.run(dA, dB).C).copy()
     res = plan.run(dA, dB, faults=faults)
@@ -386,3 +390,21 @@ def test_distributed_single_rank_nccl(P, orc):
     assert cnt["blocks"] == 16 and cnt["corrected"] == 1 and cnt["clean"] == 15
     assert norm_err(host(res.C), orc.gemm(A, B), A, B) <= 1e-13
     dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("bs", [8, 16, 32, 64])
+def test_fused_reference_sums(P, orc, bs):
+    """The epilogue reference sums equal the definition (Eq 4) up to summation order."""
+    M, N, K = 320, 192, 300
+    A = gen("uniform", M, K, 31, 0)
+    B = gen("uniform", K, N, 31, 1)
+    plan = P.ProtectedGemm(M, N, K, dtype=torch.float64, bs=bs, p=2)
+    res = plan.run(to_dev(A), to_dev(B))
+    torch.cuda.synchronize()
+    C = host(res.C)
+    Rcol = C.reshape(M // bs, bs, N).sum(axis=1)
+    Rrow = C.reshape(M, N // bs, bs).sum(axis=2)
+    scale = np.abs(C).max() * bs
+    assert np.max(np.abs(host(plan.Rcol) - Rcol)) <= 1e-14 * scale
+    assert np.max(np.abs(host(plan.Rrow) - Rrow)) <= 1e-14 * scale
+    assert res.counts()["checks_critical"] == 0
