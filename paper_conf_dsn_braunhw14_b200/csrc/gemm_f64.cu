@@ -219,14 +219,15 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
   // (a bijection of [0,16); the same permutation for A and B leaves the product unchanged).
   // With the 128B-swizzled A tile and the 64B-swizzled B boxes every half-warp of a 64-bit
   // LDS touches 16 distinct 8-byte bank slots (conflict-free: 2 wavefronts).
-  uint32_t offA[4], offB[4];
-#pragma unroll
-  for (int ks = 0; ks < 4; ++ks) {
+  // (offsets recomputed per load: cheaper than holding 8 registers across the k-loop)
+  auto offA = [&](int ks) -> uint32_t {
     const int k = (tig & 1) | ((ks & 1) << 1) | ((((tig >> 1) ^ (ks >> 1)) & 1) << 2) | ((tig >> 1) << 3);
-    offA[ks] = (uint32_t)(((wm * 32 + g) * 16 + ((((k >> 1) ^ g) << 1) | (k & 1))) * 8);
-    offB[ks] = (uint32_t)(A_BYTES + wn * 4 * 1024 +
-                          (k * 8 + ((((g >> 1) ^ ((k >> 1) & 3)) << 1) | (g & 1))) * 8);
-  }
+    return (uint32_t)(((wm * 32 + g) * 16 + ((((k >> 1) ^ g) << 1) | (k & 1))) * 8);
+  };
+  auto offB = [&](int ks) -> uint32_t {
+    const int k = (tig & 1) | ((ks & 1) << 1) | ((((tig >> 1) ^ (ks >> 1)) & 1) << 2) | ((tig >> 1) << 3);
+    return (uint32_t)(A_BYTES + wn * 4 * 1024 + (k * 8 + ((((g >> 1) ^ ((k >> 1) & 3)) << 1) | (g & 1))) * 8);
+  };
 
   double acc[MT][NT][4];
   int j = 0;
@@ -273,32 +274,44 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
 #pragma unroll
         for (int q = 0; q < 4; ++q) acc[i][jj][q] = 0.0;
 
+    // Fragments are double-buffered in registers across k4-steps AND across k-tiles: the
+    // ks = 0 fragments of k-tile kt+1 are loaded (after its full barrier) while the ks = 3
+    // DMMAs of k-tile kt issue, so no warp idles on LDS latency at a k-tile boundary.
+    double a[2][MT][2], b[2][NT];
+    auto load = [&](const uint8_t *st, int buf, int ks) {
+#pragma unroll
+      for (int mt = 0; mt < MT; ++mt) {
+        a[buf][mt][0] = *reinterpret_cast<const double *>(st + offA(ks) + mt * 2048);
+        a[buf][mt][1] = *reinterpret_cast<const double *>(st + offA(ks) + mt * 2048 + 1024);
+      }
+#pragma unroll
+      for (int nt = 0; nt < NT; ++nt)
+        b[buf][nt] = *reinterpret_cast<const double *>(st + offB(ks) + nt * 1024);
+    };
+    {
+      const int s0 = j % STAGES;
+      mbar_wait(&full[s0], (uint32_t)((j / STAGES) & 1));
+      load(smem + s0 * STAGE_BYTES, 0, 0);
+    }
     for (int kt = kt0; kt < kt_end; ++kt, ++j) {
       const int s = j % STAGES;
-      mbar_wait(&full[s], (uint32_t)((j / STAGES) & 1));
       const uint8_t *st = smem + s * STAGE_BYTES;
-      double a[2][MT][2], b[2][NT];
-      auto load = [&](int buf, int ks) {
-#pragma unroll
-        for (int mt = 0; mt < MT; ++mt) {
-          a[buf][mt][0] = *reinterpret_cast<const double *>(st + offA[ks] + mt * 2048);
-          a[buf][mt][1] = *reinterpret_cast<const double *>(st + offA[ks] + mt * 2048 + 1024);
-        }
-#pragma unroll
-        for (int nt = 0; nt < NT; ++nt)
-          b[buf][nt] = *reinterpret_cast<const double *>(st + offB[ks] + nt * 1024);
-      };
-      load(0, 0);
 #pragma unroll
       for (int ks = 0; ks < BK / 4; ++ks) {
-        if (ks + 1 < BK / 4) load((ks + 1) & 1, ks + 1);
+        if (ks + 1 < BK / 4) {
+          load(st, (ks + 1) & 1, ks + 1);
+        } else if (kt + 1 < kt_end) {
+          const int s1 = (j + 1) % STAGES;
+          mbar_wait(&full[s1], (uint32_t)(((j + 1) / STAGES) & 1));
+          load(smem + s1 * STAGE_BYTES, 0, 0);
+        }
 #pragma unroll
         for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
           for (int nt = 0; nt < NT; ++nt)
             dmma(acc[mt][nt], a[ks & 1][mt][0], a[ks & 1][mt][1], b[ks & 1][nt]);
       }
-      // release the stage to the producer
+      // release the stage to the producer (its last fragments were consumed by the ks = 3 DMMAs)
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[s]);
       if (nf > 0) {  // Alg 3 errorVecAdd1 at k-tile granularity
