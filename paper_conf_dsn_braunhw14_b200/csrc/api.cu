@@ -1,5 +1,6 @@
 // api.cu -- the C ABI of include/aabft.h: validation, workspace sizing, dispatch, errors.
 // No C++ exception crosses the ABI; every entry point is stream-ordered and never allocates.
+#include <algorithm>
 #include <atomic>
 #include <cmath>
 #include <cstdarg>
@@ -258,11 +259,38 @@ aabft_status aabft_correct(const aabft_config *cfg, const aabft_encoded *enc,
   AABFT_GUARD_END
 }
 
+}  // extern "C"
+
 // ------------------------------------------------------------------ host end-to-end entry point
+// Pipelined: A is split into S row slabs and B into S column panels (S <= 4, multiples of
+// lcm(bs, 64)); the S x S blocks of C are protected GEMMs of their own (every BS x BS block
+// lies in exactly one of them, so the check is unchanged).  Host->device copies run on a copy
+// stream in the order A0, B0, A1, B1, ..., the compute stream starts block (i, j) as soon as
+// A_i and B_j have landed (encode of a slab / panel runs once), and each finished C block is
+// copied back on a third stream -- PCIe in both directions overlaps the DMMA GEMMs.
 namespace {
+struct Split {
+  int S;
+  int64_t ms, ns;  // slab rows / panel cols (last may be shorter)
+};
+Split plan_split(const aabft_config *c) {
+  // slab rows: multiples of lcm(bs, 64) = max(bs, 64) (bs is a power of two); panel columns
+  // additionally keep the Bcs / Crow column offsets 16-byte aligned (4 x (N/bs) granules)
+  const int64_t unit = std::max<int64_t>(64, c->bs), unit_n = 4 * unit;
+  Split sp;
+  sp.S = (int)std::max<int64_t>(1, std::min<int64_t>(4, std::min(c->M / (4 * unit), c->N / unit_n)));
+  sp.ms = (c->M / sp.S + unit - 1) / unit * unit;
+  sp.ns = (c->N / sp.S + unit_n - 1) / unit_n * unit_n;
+  return sp;
+}
+int64_t piece(int64_t total, int64_t step, int i) {
+  const int64_t lo = step * i;
+  return lo >= total ? 0 : std::min(step, total - lo);
+}
 struct Arena {
   int64_t lda, ldb, ldc, ld_acs, ld_bcs, ld_ccol, ld_crow;
-  size_t oA, oB, oC, oAcs, oBcs, oCcol, oCrow, oRcol, oRrow, oTav, oTai, oTbv, oTbi, oRep, oCnt, oWs, total;
+  size_t oA, oB, oC, oAcs, oBcs, oCcol, oCrow, oRcol, oRrow, oTav, oTai, oTbv, oTbi, oRep, oCnt,
+      oCntAll, oWs, total;
 };
 Arena plan_arena(const aabft_config *c) {
   Arena a;
@@ -272,6 +300,7 @@ Arena plan_arena(const aabft_config *c) {
   a.lda = rnd(c->K); a.ldb = rnd(c->N); a.ldc = rnd(c->N);
   a.ld_acs = rnd(c->K); a.ld_bcs = rnd(c->N / c->bs);
   a.ld_ccol = rnd(c->N); a.ld_crow = rnd(c->N / c->bs);
+  const Split sp = plan_split(c);
   size_t o = 0;
   auto take = [&o](size_t bytes) { size_t r = o; o += r256(bytes); return r; };
   a.oA = take(c->M * a.lda * es);
@@ -281,19 +310,42 @@ Arena plan_arena(const aabft_config *c) {
   a.oBcs = take(c->K * a.ld_bcs * es);
   a.oCcol = take((c->M / c->bs) * a.ld_ccol * es);
   a.oCrow = take(c->M * a.ld_crow * es);
-  a.oRcol = take((c->M / c->bs) * c->N * 8);
-  a.oRrow = take(c->M * (c->N / c->bs) * 8);
-  a.oTav = take((c->M + c->M / c->bs) * c->p * 8);
-  a.oTai = take((c->M + c->M / c->bs) * c->p * 4);
-  a.oTbv = take((c->N + c->N / c->bs) * c->p * 8);
-  a.oTbi = take((c->N + c->N / c->bs) * c->p * 4);
-  a.oRep = take((c->M / c->bs) * (c->N / c->bs) * sizeof(aabft_block_report));
-  a.oCnt = take(sizeof(aabft_counts));
+  a.oRcol = take((c->M / c->bs) * c->N * 8 + 256 * sp.S * sp.S);
+  a.oRrow = take(c->M * (c->N / c->bs) * 8 + 256 * sp.S * sp.S);
+  a.oTav = take((c->M + c->M / c->bs) * c->p * 8 + 256 * sp.S);
+  a.oTai = take((c->M + c->M / c->bs) * c->p * 4 + 256 * sp.S);
+  a.oTbv = take((c->N + c->N / c->bs) * c->p * 8 + 256 * sp.S);
+  a.oTbi = take((c->N + c->N / c->bs) * c->p * 4 + 256 * sp.S);
+  a.oRep = take((c->M / c->bs) * (c->N / c->bs) * sizeof(aabft_block_report) + 256 * sp.S * sp.S);
+  a.oCnt = take(sizeof(aabft_counts) * sp.S * sp.S);
+  a.oCntAll = take(sizeof(aabft_counts));
   a.oWs = take(aabft_workspace_bytes(c));
   a.total = o;
   return a;
 }
+struct HostPipe {  // per-device copy streams + event pool (created once; the library's runtime)
+  cudaStream_t in = nullptr, out = nullptr;
+  cudaEvent_t ev[40];
+  bool ok = false;
+};
+HostPipe &host_pipe() {
+  static thread_local HostPipe hp[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  HostPipe &h = hp[dev & 63];
+  if (!h.ok) {
+    if (cudaStreamCreateWithFlags(&h.in, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaStreamCreateWithFlags(&h.out, cudaStreamNonBlocking) != cudaSuccess)
+      return h;
+    for (auto &e : h.ev)
+      if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return h;
+    h.ok = true;
+  }
+  return h;
+}
 }  // namespace
+
+extern "C" {
 
 size_t aabft_host_arena_bytes(const aabft_config *cfg) {
   if (validate(cfg) != AABFT_OK) return 0;
@@ -311,28 +363,97 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
   const Arena a = plan_arena(cfg);
   if (!arena || arena_bytes < a.total) { set_error("arena too small: need %zu bytes", a.total); return AABFT_EWORKSPACE; }
   if (!aligned16(arena)) { set_error("arena must be 16-byte aligned"); return AABFT_EINVAL; }
+  HostPipe &hp = host_pipe();
+  if (!hp.ok) return check_launch("copy stream / event creation");
   cudaStream_t st = (cudaStream_t)stream;
   char *base = static_cast<char *>(arena);
   const size_t es = elem_size(cfg);
-  if (cudaMemcpy2DAsync(base + a.oA, a.lda * es, A_host, cfg->K * es, cfg->K * es, cfg->M, cudaMemcpyHostToDevice, st) != cudaSuccess ||
-      cudaMemcpy2DAsync(base + a.oB, a.ldb * es, B_host, cfg->N * es, cfg->N * es, cfg->K, cudaMemcpyHostToDevice, st) != cudaSuccess)
-    return check_launch("host->device copy");
-  aabft_encoded enc{base + a.oAcs, a.ld_acs, base + a.oBcs, a.ld_bcs,
-                    reinterpret_cast<double *>(base + a.oTav), reinterpret_cast<int32_t *>(base + a.oTai),
-                    reinterpret_cast<double *>(base + a.oTbv), reinterpret_cast<int32_t *>(base + a.oTbi)};
-  aabft_product prod{base + a.oC, a.ldc, base + a.oCcol, a.ld_ccol, base + a.oCrow, a.ld_crow,
-                     reinterpret_cast<double *>(base + a.oRcol), reinterpret_cast<double *>(base + a.oRrow)};
-  auto *rep = reinterpret_cast<aabft_block_report *>(base + a.oRep);
-  auto *cnt = reinterpret_cast<aabft_counts *>(base + a.oCnt);
+  const int64_t M = cfg->M, N = cfg->N, K = cfg->K, bs = cfg->bs, p = cfg->p;
+  const Split sp = plan_split(cfg);
+  const int S = sp.S;
+  cudaEvent_t *evA = hp.ev, *evB = hp.ev + 4, *evC = hp.ev + 8;  // evC: S*S <= 16
+  cudaEvent_t evStart = hp.ev[24], evOutDone = hp.ev[25];
+  // the copy streams start after whatever the caller enqueued before this call
+  if (cudaEventRecord(evStart, st) != cudaSuccess || cudaStreamWaitEvent(hp.in, evStart, 0) != cudaSuccess ||
+      cudaStreamWaitEvent(hp.out, evStart, 0) != cudaSuccess)
+    return check_launch("pipeline start");
+  // host -> device: A0, B0, A1, B1, ...
+  for (int i = 0; i < S; ++i) {
+    const int64_t mi = piece(M, sp.ms, i), nj = piece(N, sp.ns, i);
+    if (mi > 0 && cudaMemcpy2DAsync(base + a.oA + (size_t)(i * sp.ms) * a.lda * es, a.lda * es,
+                                    static_cast<const char *>(A_host) + (size_t)(i * sp.ms) * K * es,
+                                    K * es, K * es, mi, cudaMemcpyHostToDevice, hp.in) != cudaSuccess)
+      return check_launch("host->device copy (A)");
+    cudaEventRecord(evA[i], hp.in);
+    if (nj > 0 && cudaMemcpy2DAsync(base + a.oB + (size_t)(i * sp.ns) * es, a.ldb * es,
+                                    static_cast<const char *>(B_host) + (size_t)(i * sp.ns) * es,
+                                    N * es, nj * es, K, cudaMemcpyHostToDevice, hp.in) != cudaSuccess)
+      return check_launch("host->device copy (B)");
+    cudaEventRecord(evB[i], hp.in);
+  }
   const size_t wsb = aabft_workspace_bytes(cfg);
-  if ((s = aabft_encode(cfg, base + a.oA, a.lda, base + a.oB, a.ldb, &enc, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
-  if ((s = aabft_gemm(cfg, base + a.oA, a.lda, base + a.oB, a.ldb, &enc, &prod, nullptr, 0, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
-  if ((s = aabft_check(cfg, &enc, &prod, rep, cnt, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
-  if ((s = aabft_correct(cfg, &enc, &prod, rep, cnt, stream)) != AABFT_OK) return s;
-  if (cudaMemcpy2DAsync(C_host, cfg->N * es, base + a.oC, a.ldc * es, cfg->N * es, cfg->M, cudaMemcpyDeviceToHost, st) != cudaSuccess)
-    return check_launch("device->host copy");
-  if (counts_host && cudaMemcpyAsync(counts_host, cnt, sizeof(aabft_counts), cudaMemcpyDeviceToHost, st) != cudaSuccess)
+  auto *cnt_blocks = reinterpret_cast<aabft_counts *>(base + a.oCnt);
+  // per-slab / per-panel top-p tables and per-block reference sums / reports (dense, block-major)
+  auto tav = [&](int i) { return reinterpret_cast<double *>(base + a.oTav) + (i * sp.ms + i * (sp.ms / bs)) * p; };
+  auto tai = [&](int i) { return reinterpret_cast<int32_t *>(base + a.oTai) + (i * sp.ms + i * (sp.ms / bs)) * p; };
+  auto tbv = [&](int j) { return reinterpret_cast<double *>(base + a.oTbv) + (j * sp.ns + j * (sp.ns / bs)) * p; };
+  auto tbi = [&](int j) { return reinterpret_cast<int32_t *>(base + a.oTbi) + (j * sp.ns + j * (sp.ns / bs)) * p; };
+  size_t rcol_off = 0, rrow_off = 0, rep_off = 0;
+  bool encA[4] = {false, false, false, false}, encB[4] = {false, false, false, false};
+  int nblk = 0;
+  // compute order: diagonal shells, so block (i, j) runs as soon as A_i and B_j are resident
+  for (int d = 0; d < S; ++d) {
+    for (int t = 0; t <= 2 * d; ++t) {
+      const int i = t <= d ? d : t - d - 1, j = t <= d ? t : d;
+      const int64_t mi = piece(M, sp.ms, i), nj = piece(N, sp.ns, j);
+      if (mi <= 0 || nj <= 0) continue;
+      aabft_config cb = *cfg;
+      cb.M = mi;
+      cb.N = nj;
+      const void *Ai = base + a.oA + (size_t)(i * sp.ms) * a.lda * es;
+      const void *Bj = base + a.oB + (size_t)(j * sp.ns) * es;
+      aabft_encoded enc{base + a.oAcs + (size_t)(i * sp.ms / bs) * a.ld_acs * es, a.ld_acs,
+                        base + a.oBcs + (size_t)(j * sp.ns / bs) * es, a.ld_bcs,
+                        tav(i), tai(i), tbv(j), tbi(j)};
+      if (!encA[i]) {
+        cudaStreamWaitEvent(st, evA[i], 0);
+        if ((s = aabft_encode(&cb, Ai, a.lda, nullptr, 0, &enc, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
+        encA[i] = true;
+      }
+      if (!encB[j]) {
+        cudaStreamWaitEvent(st, evB[j], 0);
+        if ((s = aabft_encode(&cb, nullptr, 0, Bj, a.ldb, &enc, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
+        encB[j] = true;
+      }
+      aabft_product prod{base + a.oC + ((size_t)(i * sp.ms) * a.ldc + (size_t)(j * sp.ns)) * es, a.ldc,
+                         base + a.oCcol + ((size_t)(i * sp.ms / bs) * a.ld_ccol + (size_t)(j * sp.ns)) * es, a.ld_ccol,
+                         base + a.oCrow + ((size_t)(i * sp.ms) * a.ld_crow + (size_t)(j * sp.ns / bs)) * es, a.ld_crow,
+                         reinterpret_cast<double *>(base + a.oRcol + rcol_off),
+                         reinterpret_cast<double *>(base + a.oRrow + rrow_off)};
+      auto *rep = reinterpret_cast<aabft_block_report *>(base + a.oRep + rep_off);
+      rcol_off += r256((size_t)(mi / bs) * nj * 8);
+      rrow_off += r256((size_t)mi * (nj / bs) * 8);
+      rep_off += r256((size_t)(mi / bs) * (nj / bs) * sizeof(aabft_block_report));
+      aabft_counts *cnt = cnt_blocks + nblk;
+      if ((s = aabft_gemm(&cb, Ai, a.lda, Bj, a.ldb, &enc, &prod, nullptr, 0, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
+      if ((s = aabft_check(&cb, &enc, &prod, rep, cnt, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
+      if ((s = aabft_correct(&cb, &enc, &prod, rep, cnt, stream)) != AABFT_OK) return s;
+      // device -> host of the finished (corrected) C block on the copy-out stream
+      cudaEventRecord(evC[nblk], st);
+      cudaStreamWaitEvent(hp.out, evC[nblk], 0);
+      if (cudaMemcpy2DAsync(static_cast<char *>(C_host) + ((size_t)(i * sp.ms) * N + (size_t)(j * sp.ns)) * es,
+                            N * es, prod.C, a.ldc * es, nj * es, mi, cudaMemcpyDeviceToHost, hp.out) != cudaSuccess)
+        return check_launch("device->host copy (C)");
+      ++nblk;
+    }
+  }
+  // global counters = sum over the blocks (SUM n, MAX max_ratio)
+  auto *cnt_all = reinterpret_cast<aabft_counts *>(base + a.oCntAll);
+  if ((s = launch_counts_sum(cnt_blocks, nblk, cnt_all, st)) != AABFT_OK) return s;
+  if (counts_host && cudaMemcpyAsync(counts_host, cnt_all, sizeof(aabft_counts), cudaMemcpyDeviceToHost, st) != cudaSuccess)
     return check_launch("counts copy");
+  cudaEventRecord(evOutDone, hp.out);
+  cudaStreamWaitEvent(st, evOutDone, 0);
   if (cudaStreamSynchronize(st) != cudaSuccess) return check_launch("stream sync");
   return AABFT_OK;
   AABFT_GUARD_END

@@ -378,6 +378,26 @@ aabft_status run_correct(const aabft_config *cfg, const CheckArgs &a, BoundParam
 
 }  // namespace
 
+// sum of per-part counters (SUM n[8], MAX max_ratio) -- used by the pipelined host entry point
+__global__ void counts_sum_kernel(const aabft_counts *parts, int n, aabft_counts *out) {
+  const int t = threadIdx.x;
+  if (t < 8) {
+    long long v = 0;
+    for (int i = 0; i < n; ++i) v += parts[i].n[t];
+    out->n[t] = v;
+  } else if (t == 8) {
+    double m = 0.0;
+    for (int i = 0; i < n; ++i) m = fmax(m, parts[i].max_ratio);
+    out->max_ratio = m;
+  }
+}
+
+aabft_status launch_counts_sum(const aabft_counts *parts, int n, aabft_counts *out, cudaStream_t st) {
+  counts_sum_kernel<<<1, 32, 0, st>>>(parts, n, out);
+  next_launch();
+  return check_launch("counts sum");
+}
+
 aabft_status launch_bound(const aabft_config *cfg, const aabft_encoded *enc, double *eps_col,
                           double *sig_col, double *eps_row, double *sig_row, cudaStream_t st) {
   const BoundParams bp = make_bound_params(cfg);

@@ -48,6 +48,7 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
                              const aabft_product *out, const aabft_fault *faults,
                              int32_t nfaults, bool plain, void *ws, cudaStream_t st);
 size_t encode_ws_bytes(const aabft_config *cfg);
+aabft_status launch_counts_sum(const aabft_counts *parts, int n, aabft_counts *out, cudaStream_t st);
 size_t gemm_f64_ws_bytes();
 aabft_status launch_gemm_f32(const aabft_config *cfg, const void *A, int64_t lda,
                              const void *B, int64_t ldb, const aabft_encoded *enc,

@@ -313,11 +313,13 @@ def test_multi_fault_block_uncorrectable(P, orc):
     assert res.counts()["uncorrectable"] == 1
 
 
-def test_host_entry_point_e2e(P, orc):
-    """aabft_protected_gemm_host: host buffers in, corrected C + counts out."""
+@pytest.mark.parametrize("M,N,K,bs", [(256, 128, 200, 64), (1024, 1024, 256, 64),
+                                     (1088, 1216, 130, 64), (1024, 2048, 64, 32)])
+def test_host_entry_point_e2e(P, orc, M, N, K, bs):
+    """aabft_protected_gemm_host: host buffers in, corrected C + counts out (pipelined S x S
+    blocks with overlapped copies when M, N are large enough)."""
     import ctypes as C
     from paper_conf_dsn_braunhw14_b200 import _abi
-    M, N, K, bs = 256, 128, 200, 64
     A = gen("uniform", M, K, 15, 0)
     B = gen("uniform", K, N, 15, 1)
     cfg = _abi.Config(0, bs, M, N, K, 2, 0, 3.0, 1, 0)
