@@ -1,21 +1,26 @@
 // gemm_f32.cu -- step 2 of A-ABFT (Eq 3) for FP32 on the FFMA pipe (no TF32: a
 // tensor-core TF32 product would change the rounding model the bound assumes, north_star).
 //
-// B200 design: 128 x 128 x 8 CTA tiles, 256 threads, 8 x 8 register
-// micro-tiles split 2 x 2 (rows ty*4 / 64+ty*4, cols tx*4 / 64+tx*4) so every shared-memory
-// read is an LDS.128 broadcast or a contiguous row.  Global -> register prefetch of the next
-// k-tile overlaps the 512 FFMAs of the current one (register double buffering, one barrier per
-// k-tile).  Every element accumulates c = fma(a_k, b_k, c) in ascending k, which is exactly
-// the fused sequential inner product of Eq 15 / §IV-D -- the FP32 product is bit-identical
-// to the definition.  Same three tile types as the FP64 kernel (C, Ccol, Crow) and the same
-// fault hooks (site 1 at k-tile granularity, BK = 8).
+// B200 design: 128 x 128 x 16 CTA tiles, 256 threads, 8 x 8 register
+// micro-tiles split 2 x 2 (rows ty*4 / 64+ty*4, cols tx*4 / 64+tx*4), a 3-stage cp.async
+// (LDGSTS) shared-memory ring, LDS.128 fragments and sm_100 FFMA2 (packed fp32x2 FMA).  Every
+// element accumulates c = fma(a_k, b_k, c) in ascending k, which is exactly the fused
+// sequential inner product of Eq 15 / §IV-D -- the FP32 product is bit-identical to the
+// definition.  Same three tile types as the FP64 kernel (C, Ccol, Crow) and the same fault
+// hooks (site 1 at k-tile granularity, BK = 16).
 #include "common.cuh"
 
 namespace aabft {
 namespace {
 
-constexpr int BM = 128, BN = 128, BK = 8, THREADS = 256, AST = BM + 4;
-constexpr int MAXF = 256;  // faults per 128x128 tile kept in smem (one per 8x8 block)
+#ifndef AABFT_F32_BN
+#define AABFT_F32_BN 128
+#endif
+constexpr int BM = 128, BN = AABFT_F32_BN, BK = 16, STAGES = 3;
+constexpr int TX = BN / 8, THREADS = 16 * TX;   // 16 x TX threads, 8 x 8 outputs each
+constexpr int HN = BN / 2;                      // column offset of the second 4-wide half
+constexpr int MAXF = BM * BN / 64;  // faults per tile kept in smem (one per 8x8 block)
+constexpr int SMEM32 = STAGES * (BM + BN) * BK * 4 + MAXF * (int)sizeof(aabft_fault);
 constexpr int GROUP_M = 8;
 
 struct SgemmArgs {
@@ -40,28 +45,29 @@ struct SgemmArgs {
   int nfaults;
 };
 
-__device__ __forceinline__ float4 load4(const float *base, int64_t ld, int64_t r, int64_t rows,
-                                        int64_t c, int64_t cols) {
-  if (r < rows && c + 3 < cols) return __ldg(reinterpret_cast<const float4 *>(base + r * ld + c));
-  float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-  if (r < rows) {
-    const float *p = base + r * ld;
-    if (c < cols) v.x = __ldg(p + c);
-    if (c + 1 < cols) v.y = __ldg(p + c + 1);
-    if (c + 2 < cols) v.z = __ldg(p + c + 2);
-    if (c + 3 < cols) v.w = __ldg(p + c + 3);
-  }
-  return v;
-}
-
 __device__ __forceinline__ float xor_bits(float v, uint64_t m) {
   return __int_as_float(__float_as_int(v) ^ (int)(uint32_t)m);
 }
 
+// 16-byte cp.async (LDGSTS) with zero-fill of the bytes beyond `valid` (0..16)
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem, int valid) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(smem)),
+               "l"(gmem), "r"(valid)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
 __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs args) {
-  __shared__ __align__(16) float As[2][BK][AST];
-  __shared__ __align__(16) float Bs[2][BK][BN];
-  __shared__ aabft_fault s_f[MAXF];
+  // 3-stage cp.async ring: A tile [128 rows][16 k] (k contiguous, as in memory), B tile
+  // [16 k][128 cols].  A fragments are LDS.128 along k (4 k-steps of one row), B fragments
+  // LDS.128 along n; the 8 x 8 micro-tile runs as 32 FFMA2 per k-step (sm_100 packed fp32x2
+  // FMA, A broadcast) -- each lane rounded once, exactly fmaf.
+  extern __shared__ __align__(16) uint8_t smem32[];
+  auto As = reinterpret_cast<float(*)[BM][BK]>(smem32);                          // [STAGES]
+  auto Bs = reinterpret_cast<float(*)[BK][BN]>(smem32 + STAGES * BM * BK * 4);   // [STAGES]
+  aabft_fault *s_f = reinterpret_cast<aabft_fault *>(smem32 + STAGES * (BM + BN) * BK * 4);
   __shared__ int s_nf;
 
   int64_t bid = blockIdx.x;
@@ -95,9 +101,7 @@ __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs ar
   const int64_t cols_valid = type == 2 ? args.Ncs : args.N;
   const int64_t K = args.K;
 
-  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
-  const int a_row = tid >> 1, a_k = (tid & 1) * 4;
-  const int b_k = tid >> 5, b_n = (tid & 31) * 4;
+  const int tid = threadIdx.x, tx = tid % TX, ty = tid / TX;
 
   int nf = 0;
   if (args.nfaults > 0) {
@@ -124,41 +128,67 @@ __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs ar
     nf = min(s_nf, MAXF);
   }
 
-  float acc[8][8];
+  // tile loaders: 2 x 16-byte chunks of A and of B per thread per k-tile
+  auto load_tile = [&](int stage, int kt) {
+    const int64_t k0 = (int64_t)kt * BK;
+#pragma unroll
+    for (int c = 0; c < BM * BK / 4 / THREADS; ++c) {
+      const int e = tid + c * THREADS;
+      const int ar = e >> 2, ak = (e & 3) * 4;   // A: row ar, k ak..ak+3
+      const int64_t gr = m0 + ar, gk = k0 + ak;
+      const int av = (gr < rows_valid && gk < K) ? (int)((K - gk) * 4 < 16 ? (K - gk) * 4 : 16) : 0;
+      cp_async16(&As[stage][ar][ak], av ? (const void *)(Ap + gr * lda + gk) : (const void *)Ap, av);
+    }
+#pragma unroll
+    for (int c = 0; c < BK * BN / 4 / THREADS; ++c) {
+      const int e = tid + c * THREADS;
+      const int bk = e / (BN / 4), bn = (e % (BN / 4)) * 4;  // B: k row bk, cols bn..bn+3
+      const int64_t gkb = k0 + bk, gn = n0 + bn;
+      const int bv = (gkb < K && gn < cols_valid) ? (int)((cols_valid - gn) * 4 < 16 ? (cols_valid - gn) * 4 : 16) : 0;
+      cp_async16(&Bs[stage][bk][bn], bv ? (const void *)(Bp + gkb * ldb + gn) : (const void *)Bp, bv);
+    }
+  };
+
+  float2 acc2[8][4];
 #pragma unroll
   for (int i = 0; i < 8; ++i)
 #pragma unroll
-    for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
+    for (int j = 0; j < 4; ++j) acc2[i][j] = make_float2(0.f, 0.f);
+#define ACC(i, j) (((j) & 1) ? acc2[i][(j) >> 1].y : acc2[i][(j) >> 1].x)
 
   const int nk = (int)((K + BK - 1) / BK);
-  float4 ra = load4(Ap, lda, m0 + a_row, rows_valid, a_k, K);
-  float4 rb = load4(Bp, ldb, b_k, K, n0 + b_n, cols_valid);
-  As[0][a_k + 0][a_row] = ra.x;
-  As[0][a_k + 1][a_row] = ra.y;
-  As[0][a_k + 2][a_row] = ra.z;
-  As[0][a_k + 3][a_row] = ra.w;
-  *reinterpret_cast<float4 *>(&Bs[0][b_k][b_n]) = rb;
-  __syncthreads();
-
+#pragma unroll
+  for (int st = 0; st < STAGES - 1; ++st) {
+    if (st < nk) load_tile(st, st);
+    cp_async_commit();
+  }
   for (int kt = 0; kt < nk; ++kt) {
-    const int cur = kt & 1;
-    if (kt + 1 < nk) {
-      const int64_t k0 = (int64_t)(kt + 1) * BK;
-      ra = load4(Ap, lda, m0 + a_row, rows_valid, k0 + a_k, K);
-      rb = load4(Bp, ldb, k0 + b_k, K, n0 + b_n, cols_valid);
-    }
+    cp_async_wait<STAGES - 2>();
+    __syncthreads();  // tile kt visible to all; the stage consumed at kt-1 is free
+    if (kt + STAGES - 1 < nk) load_tile((kt + STAGES - 1) % STAGES, kt + STAGES - 1);
+    cp_async_commit();
+    const int cur = kt % STAGES;
 #pragma unroll
-    for (int k = 0; k < BK; ++k) {
-      const float4 a0 = *reinterpret_cast<const float4 *>(&As[cur][k][ty * 4]);
-      const float4 a1 = *reinterpret_cast<const float4 *>(&As[cur][k][64 + ty * 4]);
-      const float4 b0 = *reinterpret_cast<const float4 *>(&Bs[cur][k][tx * 4]);
-      const float4 b1 = *reinterpret_cast<const float4 *>(&Bs[cur][k][64 + tx * 4]);
-      const float av[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
-      const float bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+    for (int k4 = 0; k4 < BK / 4; ++k4) {
+      float4 a4[8];
 #pragma unroll
-      for (int i = 0; i < 8; ++i)
+      for (int i = 0; i < 8; ++i) {
+        const int r = i < 4 ? ty * 4 + i : 64 + ty * 4 + (i - 4);
+        a4[i] = *reinterpret_cast<const float4 *>(&As[cur][r][k4 * 4]);
+      }
 #pragma unroll
-        for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
+      for (int kk = 0; kk < 4; ++kk) {
+        const float4 b0 = *reinterpret_cast<const float4 *>(&Bs[cur][k4 * 4 + kk][tx * 4]);
+        const float4 b1 = *reinterpret_cast<const float4 *>(&Bs[cur][k4 * 4 + kk][HN + tx * 4]);
+        const float2 bv[4] = {make_float2(b0.x, b0.y), make_float2(b0.z, b0.w),
+                              make_float2(b1.x, b1.y), make_float2(b1.z, b1.w)};
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const float av = kk == 0 ? a4[i].x : (kk == 1 ? a4[i].y : (kk == 2 ? a4[i].z : a4[i].w));
+#pragma unroll
+          for (int j = 0; j < 4; ++j) acc2[i][j] = __ffma2_rn(make_float2(av, av), bv[j], acc2[i][j]);
+        }
+      }
     }
     if (nf > 0) {
       for (int f = 0; f < nf; ++f) {
@@ -169,21 +199,13 @@ __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs ar
 #pragma unroll
           for (int j = 0; j < 8; ++j) {
             const int r = (i < 4 ? ty * 4 + i : 64 + ty * 4 + i - 4);
-            const int c = (j < 4 ? tx * 4 + j : 64 + tx * 4 + j - 4);
-            if (r == ft.row && c == ft.col) acc[i][j] = xor_bits(acc[i][j], ft.xor_mask);
+            const int c = (j < 4 ? tx * 4 + j : HN + tx * 4 + j - 4);
+            if (r == ft.row && c == ft.col) ACC(i, j) = xor_bits(ACC(i, j), ft.xor_mask);
           }
       }
     }
-    if (kt + 1 < nk) {
-      const int nxt = cur ^ 1;
-      As[nxt][a_k + 0][a_row] = ra.x;
-      As[nxt][a_k + 1][a_row] = ra.y;
-      As[nxt][a_k + 2][a_row] = ra.z;
-      As[nxt][a_k + 3][a_row] = ra.w;
-      *reinterpret_cast<float4 *>(&Bs[nxt][b_k][b_n]) = rb;
-    }
-    __syncthreads();
   }
+  cp_async_wait<0>();
 
   if (nf > 0) {
     for (int f = 0; f < nf; ++f) {
@@ -194,10 +216,10 @@ __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs ar
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
           const int r = (i < 4 ? ty * 4 + i : 64 + ty * 4 + i - 4);
-          const int c = (j < 4 ? tx * 4 + j : 64 + tx * 4 + j - 4);
+          const int c = (j < 4 ? tx * 4 + j : HN + tx * 4 + j - 4);
           if (r == ft.row && c == ft.col)
-            acc[i][j] = ft.site == 0 ? xor_bits(acc[i][j], ft.xor_mask)
-                                     : (float)((double)acc[i][j] + ft.add);
+            ACC(i, j) = ft.site == 0 ? xor_bits(ACC(i, j), ft.xor_mask)
+                                     : (float)((double)ACC(i, j) + ft.add);
         }
     }
   }
@@ -213,18 +235,19 @@ __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs ar
     if (r >= rows_valid) continue;
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
-      const int64_t c = n0 + h * 64 + tx * 4;
+      const int64_t c = n0 + h * HN + tx * 4;
       float *p = out + r * ld + c;
       if (c + 3 < cols_valid && vec_ok) {
         *reinterpret_cast<float4 *>(p) =
-            make_float4(acc[i][h * 4], acc[i][h * 4 + 1], acc[i][h * 4 + 2], acc[i][h * 4 + 3]);
+            make_float4(ACC(i, h * 4), ACC(i, h * 4 + 1), ACC(i, h * 4 + 2), ACC(i, h * 4 + 3));
       } else {
 #pragma unroll
         for (int j = 0; j < 4; ++j)
-          if (c + j < cols_valid) p[j] = acc[i][h * 4 + j];
+          if (c + j < cols_valid) p[j] = ACC(i, h * 4 + j);
       }
     }
   }
+#undef ACC
 }
 
 }  // namespace
@@ -259,8 +282,14 @@ aabft_status launch_gemm_f32(const aabft_config *cfg, const void *A, int64_t lda
   a.faults = faults;
   a.nfaults = faults ? nfaults : 0;
   const int64_t tiles = a.n0 + a.n1 + a.n2;
+  static bool attr = false;
+  if (!attr) {
+    if (cudaFuncSetAttribute(gemm_f32_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM32) != cudaSuccess)
+      return check_launch("gemm_f32 smem attribute");
+    attr = true;
+  }
   if (tiles > 0) {
-    gemm_f32_kernel<<<(unsigned)tiles, THREADS, 0, st>>>(a);
+    gemm_f32_kernel<<<(unsigned)tiles, THREADS, SMEM32, st>>>(a);
     next_launch();
   }
   return check_launch("aabft_gemm(f32)");
