@@ -103,7 +103,7 @@ static aabft_status device_ok() {
 
 // rows of a row-major operand fed to TMA / vector loads: base 16-B aligned, pitch 16-B multiple
 static size_t gemm_ws_bytes(const aabft_config *c) {
-  return c->dtype == AABFT_F64 ? gemm_f64_ws_bytes() : 0;
+  return c->dtype == AABFT_F64 ? gemm_f64_ws_bytes(c) : 0;
 }
 static void *gemm_ws(const aabft_config *c, void *ws) {
   return static_cast<char *>(ws) + r256(encode_ws_bytes(c));
@@ -241,11 +241,15 @@ aabft_status aabft_check(const aabft_config *cfg, const aabft_encoded *enc,
                          const aabft_product *prod, aabft_block_report *reports,
                          aabft_counts *counts, void *ws, size_t ws_bytes, void *stream) {
   AABFT_GUARD_BEGIN
-  (void)ws;
-  (void)ws_bytes;
   aabft_status s = check_common(cfg, enc, prod, reports, counts);
   if (s != AABFT_OK) return s;
-  return launch_check(cfg, enc, prod, reports, counts, (cudaStream_t)stream);
+  const bool fused = prod->Rcol && prod->Rrow && cfg->dtype == AABFT_F64 && cfg->bs <= 64;
+  if (fused && (!ws || ws_bytes < aabft_workspace_bytes(cfg))) {
+    set_error("check (fused): the aabft_gemm workspace is required");
+    return AABFT_EWORKSPACE;
+  }
+  return launch_check(cfg, enc, prod, reports, counts, fused ? gemm_ws(cfg, ws) : nullptr,
+                      (cudaStream_t)stream);
   AABFT_GUARD_END
 }
 

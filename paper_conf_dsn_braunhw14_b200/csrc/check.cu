@@ -120,6 +120,8 @@ struct CheckArgs {
   aabft_counts *cnt;
   const double *Rcol;  // fused reference sums from the GEMM epilogue (NULL = re-sum C)
   const double *Rrow;
+  const double *Rcol2;  // BS = 64: second partials (wm = 1 / wn = 1 warps), added in order
+  const double *Rrow2;
 };
 
 // block verdict + report + aggregated counter update (shared by both check kernels)
@@ -247,7 +249,12 @@ __global__ void __launch_bounds__(128) check_fused_kernel(CheckArgs a, BoundPara
     Bound b;
     if (e < bs) {  // column check j
       const int64_t j = J * bs + e;
-      d = a.Rcol[I * a.N + j] - (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
+      double ref = a.Rcol[I * a.N + j];
+      if (bs == 64) {  // complete the two epilogue halves (and leave the full sum in Rcol)
+        ref = ref + a.Rcol2[I * a.N + j];
+        const_cast<double *>(a.Rcol)[I * a.N + j] = ref;
+      }
+      d = ref - (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
       b = bound_of(bp, y_bound<P>(a.tav + (a.M + I) * P, a.tai + (a.M + I) * P, a.tbv + j * P,
                                   a.tbi + j * P));
       const int cl = classify(d, b);
@@ -255,7 +262,12 @@ __global__ void __launch_bounds__(128) check_fused_kernel(CheckArgs a, BoundPara
       if (cl == 2) { atomicAdd(&s_nc, 1); s_col = (int)j; }
     } else {  // row check i
       const int64_t i = I * bs + (e - bs);
-      d = a.Rrow[i * nJ + J] - (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
+      double ref = a.Rrow[i * nJ + J];
+      if (bs == 64) {
+        ref = ref + a.Rrow2[i * nJ + J];
+        const_cast<double *>(a.Rrow)[i * nJ + J] = ref;
+      }
+      d = ref - (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
       b = bound_of(bp, y_bound<P>(a.tav + i * P, a.tai + i * P, a.tbv + (a.N + J) * P,
                                   a.tbi + (a.N + J) * P));
       const int cl = classify(d, b);
@@ -316,7 +328,7 @@ __global__ void correct_kernel(CheckArgs a, BoundParams bp, T *C) {
 }
 
 CheckArgs make_args(const aabft_config *cfg, const aabft_encoded *enc, const aabft_product *prod,
-                    aabft_block_report *rep, aabft_counts *cnt) {
+                    aabft_block_report *rep, aabft_counts *cnt, void *gemm_ws = nullptr) {
   CheckArgs a;
   a.M = cfg->M; a.N = cfg->N; a.bs = cfg->bs;
   a.C = prod->C; a.ldc = prod->ldc;
@@ -327,8 +339,15 @@ CheckArgs make_args(const aabft_config *cfg, const aabft_encoded *enc, const aab
   a.rep = rep; a.cnt = cnt;
   // fused reference sums exist only where aabft_gemm produces them (FP64, bs <= 64)
   const bool fused = prod->Rcol && prod->Rrow && cfg->dtype == AABFT_F64 && cfg->bs <= 64;
-  a.Rcol = fused ? prod->Rcol : nullptr;
-  a.Rrow = fused ? prod->Rrow : nullptr;
+  a.Rcol = fused && gemm_ws ? prod->Rcol : nullptr;
+  a.Rrow = fused && gemm_ws ? prod->Rrow : nullptr;
+  a.Rcol2 = a.Rrow2 = nullptr;
+  if (a.Rcol) {
+    double *rc2, *rr2;
+    gemm_f64_red_ptrs(cfg, gemm_ws, &rc2, &rr2);
+    a.Rcol2 = rc2;
+    a.Rrow2 = rr2;
+  }
   return a;
 }
 
@@ -416,9 +435,9 @@ aabft_status launch_bound(const aabft_config *cfg, const aabft_encoded *enc, dou
 
 aabft_status launch_check(const aabft_config *cfg, const aabft_encoded *enc,
                           const aabft_product *prod, aabft_block_report *rep, aabft_counts *cnt,
-                          cudaStream_t st) {
+                          void *gemm_ws, cudaStream_t st) {
   const BoundParams bp = make_bound_params(cfg);
-  const CheckArgs a = make_args(cfg, enc, prod, rep, cnt);
+  const CheckArgs a = make_args(cfg, enc, prod, rep, cnt, gemm_ws);
   if (cudaMemsetAsync(cnt, 0, sizeof(aabft_counts), st) != cudaSuccess)
     return check_launch("aabft_check memset");
   if (cfg->dtype == AABFT_F64) {

@@ -49,14 +49,15 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
                              int32_t nfaults, bool plain, void *ws, cudaStream_t st);
 size_t encode_ws_bytes(const aabft_config *cfg);
 aabft_status launch_counts_sum(const aabft_counts *parts, int n, aabft_counts *out, cudaStream_t st);
-size_t gemm_f64_ws_bytes();
+size_t gemm_f64_ws_bytes(const aabft_config *cfg);
+void gemm_f64_red_ptrs(const aabft_config *cfg, void *gemm_ws, double **rcol2, double **rrow2);
 aabft_status launch_gemm_f32(const aabft_config *cfg, const void *A, int64_t lda,
                              const void *B, int64_t ldb, const aabft_encoded *enc,
                              const aabft_product *out, const aabft_fault *faults,
                              int32_t nfaults, bool plain, cudaStream_t st);
 aabft_status launch_check(const aabft_config *cfg, const aabft_encoded *enc,
                           const aabft_product *prod, aabft_block_report *rep,
-                          aabft_counts *cnt, cudaStream_t st);
+                          aabft_counts *cnt, void *gemm_ws, cudaStream_t st);
 aabft_status launch_correct(const aabft_config *cfg, const aabft_encoded *enc,
                             const aabft_product *prod, aabft_block_report *rep,
                             aabft_counts *cnt, cudaStream_t st);

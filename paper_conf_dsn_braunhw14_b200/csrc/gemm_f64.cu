@@ -51,9 +51,8 @@ constexpr int B_BYTES = BK * TILE * 8;      // 8 KiB
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 constexpr int MAXF = 64;                    // faults per 64x64 tile kept in smem (one per 8x8 block)
 constexpr int BOOK = 128;                   // barriers, counters, cursor
-constexpr int RED_BYTES = 2 * 2 * 32 * 8;  // cross-warp partial reference sums (BS = 64)
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + BOOK +
-                           MAXF * (int)sizeof(aabft_fault) + RED_BYTES;
+                           MAXF * (int)sizeof(aabft_fault);
 constexpr int GROUP_M = AABFT_F64_GROUP_M;
 constexpr int kMaxCtas = 1024;              // >= resident CTAs; sizes the split-K partial slots
 constexpr int ACC = MT * NT * 4;            // accumulators per thread
@@ -77,6 +76,8 @@ struct GemmArgs {
   int nfaults;
   double *Rcol;                       // fused reference sums (NULL = unfused): (M/bs) x N
   double *Rrow;                       //                                         M x (N/bs)
+  double *Rcol2;                      // BS = 64: partials of the wm = 1 warps (workspace)
+  double *Rrow2;                      //          partials of the wn = 1 warps (workspace)
   int bs;
 };
 
@@ -158,8 +159,6 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
   int *s_nf = reinterpret_cast<int *>(empty + STAGES);
   static_assert(16 * STAGES + 8 <= BOOK, "bookkeeping fits");
   aabft_fault *s_f = reinterpret_cast<aabft_fault *>(smem + STAGES * STAGE_BYTES + BOOK);
-  double *s_red = reinterpret_cast<double *>(smem + STAGES * STAGE_BYTES + BOOK +
-                                             MAXF * sizeof(aabft_fault));  // [2][2][32]
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int g = lane >> 2, tig = lane & 3;
@@ -466,40 +465,28 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
             }
           }
         }
-      if (bs == 64) {  // the whole tile is one block: combine the 2 x 2 warps via smem
-        double *s_col = s_red;       // [wn][32]: column partials of the wm = 1 warps
-        double *s_row = s_red + 64;  // [wm][32]: row partials of the wn = 1 warps
-        mma_sync_bar();
-        if (wm == 1 && g == 0) {
-#pragma unroll
-          for (int nt = 0; nt < NT; ++nt)
-#pragma unroll
-            for (int e = 0; e < 2; ++e) s_col[wn * 32 + nt * 8 + tig * 2 + e] = csum[nt][e];
-        }
-        if (wn == 1 && tig == 0) {
-#pragma unroll
-          for (int mt = 0; mt < MT; ++mt)
-#pragma unroll
-            for (int h = 0; h < 2; ++h) s_row[wm * 32 + mt * 16 + h * 8 + g] = rsum[mt][h];
-        }
-        mma_sync_bar();
+      if (bs == 64) {  // the whole tile is one block: each half-warp-grid writes its own
+        // partial (no inter-warp barrier in the epilogue); aabft_check adds the two halves in
+        // a fixed order (wm = 0 + wm = 1, wn = 0 + wn = 1)
         const int64_t I = (int64_t)tl.m0 / 64, J = (int64_t)tl.n0 / 64;
-        if (wm == 0 && g == 0) {
+        double *rc = wm == 0 ? args.Rcol : args.Rcol2;
+        double *rr = wn == 0 ? args.Rrow : args.Rrow2;
+        if (g == 0) {
 #pragma unroll
           for (int nt = 0; nt < NT; ++nt)
 #pragma unroll
             for (int e = 0; e < 2; ++e) {
-              const int c = wn * 32 + nt * 8 + tig * 2 + e;
-              if (tl.n0 + c < args.N) args.Rcol[I * args.N + tl.n0 + c] = csum[nt][e] + s_col[c];
+              const int64_t c = cbase + nt * 8 + tig * 2 + e;
+              if (c < args.N) rc[I * args.N + c] = csum[nt][e];
             }
         }
-        if (wn == 0 && tig == 0) {
+        if (tig == 0) {
 #pragma unroll
           for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
-              const int r = wm * 32 + mt * 16 + h * 8 + g;
-              if (tl.m0 + r < args.M) args.Rrow[((int64_t)tl.m0 + r) * nJ + J] = rsum[mt][h] + s_row[r];
+              const int64_t r = rbase + mt * 16 + h * 8 + g;
+              if (r < args.M) rr[r * nJ + J] = rsum[mt][h];
             }
         }
       }
@@ -570,8 +557,18 @@ bool make_map(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer, 
 
 }  // namespace
 
-size_t gemm_f64_ws_bytes() {
-  return (size_t)kMaxCtas * ACC * THREADS * sizeof(double) + kMaxCtas * sizeof(int) + 256;
+static size_t r256z(size_t b) { return (b + 255) / 256 * 256; }
+static size_t red_off() {
+  return r256z((size_t)kMaxCtas * ACC * THREADS * sizeof(double) + kMaxCtas * sizeof(int));
+}
+size_t gemm_f64_ws_bytes(const aabft_config *cfg) {
+  return red_off() + r256z((size_t)(cfg->M / cfg->bs) * cfg->N * 8) +
+         r256z((size_t)cfg->M * (cfg->N / cfg->bs) * 8) + 256;
+}
+void gemm_f64_red_ptrs(const aabft_config *cfg, void *ws, double **rcol2, double **rrow2) {
+  char *w = static_cast<char *>(ws) + red_off();
+  *rcol2 = reinterpret_cast<double *>(w);
+  *rrow2 = reinterpret_cast<double *>(w + r256z((size_t)(cfg->M / cfg->bs) * cfg->N * 8));
 }
 
 aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
@@ -631,6 +628,7 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
   const bool fused = !plain && out->Rcol && out->Rrow && bs <= TILE;
   a.Rcol = fused ? out->Rcol : nullptr;
   a.Rrow = fused ? out->Rrow : nullptr;
+  gemm_f64_red_ptrs(cfg, ws, &a.Rcol2, &a.Rrow2);
 
   CUtensorMap tA, tAcs, tB, tBcs;
   if (!make_map(&tA, A, K, M, lda, BK, TILE, CU_TENSOR_MAP_SWIZZLE_128B)) return AABFT_EINVAL;

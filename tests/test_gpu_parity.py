@@ -396,7 +396,8 @@ def test_distributed_single_rank_nccl(P, orc):
 
 @pytest.mark.parametrize("bs", [8, 16, 32, 64])
 def test_fused_reference_sums(P, orc, bs):
-    """The epilogue reference sums equal the definition (Eq 4) up to summation order."""
+    """The epilogue reference sums (completed by aabft_check) equal the definition (Eq 4) up to
+    summation order."""
     M, N, K = 320, 192, 300
     A = gen("uniform", M, K, 31, 0)
     B = gen("uniform", K, N, 31, 1)
