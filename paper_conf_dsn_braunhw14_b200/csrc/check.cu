@@ -120,8 +120,9 @@ struct CheckArgs {
   aabft_counts *cnt;
   const double *Rcol;  // fused reference sums from the GEMM epilogue (NULL = re-sum C)
   const double *Rrow;
-  const double *Rcol2;  // BS = 64: second partials (wm = 1 / wn = 1 warps), added in order
-  const double *Rrow2;
+  const double *Rcol2;  // further partial reference sums from the epilogue, added in order
+  const double *Rrow2;  // (Rrow2 holds row_parts - 1 planes of M x N/bs)
+  int col_parts, row_parts;
 };
 
 // block verdict + report + aggregated counter update (shared by both check kernels)
@@ -250,7 +251,7 @@ __global__ void __launch_bounds__(128) check_fused_kernel(CheckArgs a, BoundPara
     if (e < bs) {  // column check j
       const int64_t j = J * bs + e;
       double ref = a.Rcol[I * a.N + j];
-      if (bs == 64) {  // complete the two epilogue halves (and leave the full sum in Rcol)
+      if (a.col_parts > 1) {  // complete the epilogue parts (and leave the full sum in Rcol)
         ref = ref + a.Rcol2[I * a.N + j];
         const_cast<double *>(a.Rcol)[I * a.N + j] = ref;
       }
@@ -263,8 +264,8 @@ __global__ void __launch_bounds__(128) check_fused_kernel(CheckArgs a, BoundPara
     } else {  // row check i
       const int64_t i = I * bs + (e - bs);
       double ref = a.Rrow[i * nJ + J];
-      if (bs == 64) {
-        ref = ref + a.Rrow2[i * nJ + J];
+      if (a.row_parts > 1) {
+        for (int q = 1; q < a.row_parts; ++q) ref = ref + a.Rrow2[(q - 1) * a.M * nJ + i * nJ + J];
         const_cast<double *>(a.Rrow)[i * nJ + J] = ref;
       }
       d = ref - (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
@@ -342,7 +343,9 @@ CheckArgs make_args(const aabft_config *cfg, const aabft_encoded *enc, const aab
   a.Rcol = fused && gemm_ws ? prod->Rcol : nullptr;
   a.Rrow = fused && gemm_ws ? prod->Rrow : nullptr;
   a.Rcol2 = a.Rrow2 = nullptr;
+  a.col_parts = a.row_parts = 1;
   if (a.Rcol) {
+    a.col_parts = gemm_f64_fused_parts(cfg->bs, &a.row_parts);
     double *rc2, *rr2;
     gemm_f64_red_ptrs(cfg, gemm_ws, &rc2, &rr2);
     a.Rcol2 = rc2;

@@ -51,6 +51,7 @@ size_t encode_ws_bytes(const aabft_config *cfg);
 aabft_status launch_counts_sum(const aabft_counts *parts, int n, aabft_counts *out, cudaStream_t st);
 size_t gemm_f64_ws_bytes(const aabft_config *cfg);
 void gemm_f64_red_ptrs(const aabft_config *cfg, void *gemm_ws, double **rcol2, double **rrow2);
+int gemm_f64_fused_parts(int bs, int *row_parts);  // returns column parts
 aabft_status launch_gemm_f32(const aabft_config *cfg, const void *A, int64_t lda,
                              const void *B, int64_t ldb, const aabft_encoded *enc,
                              const aabft_product *out, const aabft_fault *faults,

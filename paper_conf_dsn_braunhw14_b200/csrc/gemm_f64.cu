@@ -41,11 +41,19 @@ namespace {
 #define AABFT_F64_GROUP_M 16
 #endif
 constexpr int TILE = 64, BK = 16, STAGES = AABFT_F64_STAGES;
-constexpr int NCW = 4;                      // MMA warps per CTA (2 x 2)
+#ifndef AABFT_F64_NT
+#define AABFT_F64_NT 4
+#endif
+constexpr int NT = AABFT_F64_NT;            // n8 fragments per warp (warp tile 32 x 8*NT)
+constexpr int MT = 2;                       // m16 fragments per warp
+constexpr int WTN = NT * 8;                 // warp tile columns
+constexpr int WARPS_N = 64 / WTN;           // warps across the 64-column tile
+constexpr int NCW = 2 * WARPS_N;            // MMA warps per CTA (2 x WARPS_N)
 constexpr int THREADS = NCW * 32;           // MMA threads (named barrier 1)
 constexpr int CTA_THREADS = THREADS + 32;   // + 1 TMA producer warp
-constexpr int CTAS_PER_SM = 3;              // 15 warps / SM -> 128 registers each
-constexpr int MT = 2, NT = 4;               // m16 x n8 fragments per warp: 32 x 32 warp tile
+constexpr int CTAS_PER_SM = NCW == 4 ? 3 : 2;  // 15 / 18 warps per SM (128 / <= 102 registers)
+constexpr int COL_PARTS = 2;                // fused column sums: BS=64 spans the 2 warp rows
+constexpr int ROW_PARTS = 64 / WTN;         // fused row sums: BS=64 spans WARPS_N warp columns
 constexpr int A_BYTES = TILE * BK * 8;      // 8 KiB
 constexpr int B_BYTES = BK * TILE * 8;      // 8 KiB
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
@@ -162,7 +170,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int g = lane >> 2, tig = lane & 3;
-  const int wm = warp >> 1, wn = warp & 1;
+  const int wm = warp / WARPS_N, wn = warp % WARPS_N;
 
   // this CTA's k-tile sequence: its data-parallel tiles, then its stream-K slice
   const int64_t sk0 = sk_begin(args, blockIdx.x), sk1 = sk_begin(args, blockIdx.x + 1);
@@ -225,7 +233,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
   };
   auto offB = [&](int ks) -> uint32_t {
     const int k = (tig & 1) | ((ks & 1) << 1) | ((((tig >> 1) ^ (ks >> 1)) & 1) << 2) | ((tig >> 1) << 3);
-    return (uint32_t)(A_BYTES + wn * 4 * 1024 + (k * 8 + ((((g >> 1) ^ ((k >> 1) & 3)) << 1) | (g & 1))) * 8);
+    return (uint32_t)(A_BYTES + wn * NT * 1024 + (k * 8 + ((((g >> 1) ^ ((k >> 1) & 3)) << 1) | (g & 1))) * 8);
   };
 
   double acc[MT][NT][4];
@@ -237,7 +245,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
     const Tile tl = tile_of(args, tile);
     const int seg_len = min(args.nk - kt0, njobs - j);
     const int kt_end = kt0 + seg_len;  // exclusive
-    const int64_t rbase = (int64_t)tl.m0 + wm * 32, cbase = (int64_t)tl.n0 + wn * 32;
+    const int64_t rbase = (int64_t)tl.m0 + wm * 32, cbase = (int64_t)tl.n0 + wn * WTN;
 
     // faults that hit this tile (output coordinates of the tile's product)
     int nf = 0;
@@ -388,13 +396,14 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
       }
     }
     if (args.Rcol != nullptr && tl.type == 0) {
-      // ---- fused reference sums (Eq 4) of the BS x BS blocks inside this 64 x 64 C tile, taken
-      // from the registers that are about to be stored (after any injected fault), in a fixed
-      // order: 8-row/8-column shuffle trees, then pairwise over fragments, then across warps.
+      // ---- fused reference sums (Eq 4) of the BS x BS blocks touching this 64 x 64 C tile,
+      // taken from the registers about to be stored (after any injected fault), in a fixed
+      // order: 8-row / 8-column shuffle trees, then pairwise over fragments.  A block larger
+      // than the warp tile (rows > 32 or columns > WTN) is left as per-warp partials ("parts",
+      // part 0 in Rcol/Rrow, the others in the workspace) that aabft_check adds in part order.
       const int bs = args.bs;
       const int64_t nJ = args.N / bs;
-      double csum[NT][2], rsum[MT][2];  // per-warp totals (used for BS = 64)
-      // column sums: per (nt, e) column, 8-row shuffle trees then pairwise over (mt, h)
+      // column sums: per (nt, e) column, 8-row trees over g, then (h, mt) pairwise
 #pragma unroll
       for (int nt = 0; nt < NT; ++nt)
 #pragma unroll
@@ -411,9 +420,9 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
               c8[mt][h] = v;  // rows mt*16 + h*8 + (0..7)
             }
           const double c16a = c8[0][0] + c8[0][1], c16b = c8[1][0] + c8[1][1];
-          csum[nt][e] = c16a + c16b;
+          const double c32 = c16a + c16b;
           const int64_t col = cbase + nt * 8 + tig * 2 + e;
-          if (bs <= 32 && g == 0 && col < args.N) {
+          if (g == 0 && col < args.N) {
             if (bs == 8) {
 #pragma unroll
               for (int mt = 0; mt < MT; ++mt)
@@ -426,13 +435,15 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
               const int64_t I0 = rbase / 16;
               if (I0 * 16 < args.M) args.Rcol[I0 * args.N + col] = c16a;
               if ((I0 + 1) * 16 < args.M) args.Rcol[(I0 + 1) * args.N + col] = c16b;
-            } else {
-              const int64_t I = rbase / 32;
-              if (I * 32 < args.M) args.Rcol[I * args.N + col] = csum[nt][e];
+            } else {  // 32 or 64: one value per warp; part = which 32-row half of the block
+              const int64_t I = rbase / bs;
+              const int part = (int)((rbase % bs) / 32);
+              double *dst = part == 0 ? args.Rcol : args.Rcol2;
+              if (rbase < args.M) dst[I * args.N + col] = c32;
             }
           }
         }
-      // row sums: per (mt, h) row, pairwise over e, 4-lane shuffle tree, then over nt
+      // row sums: per (mt, h) row, pairwise over e, 4-lane tree over tig, then over nt
 #pragma unroll
       for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
@@ -445,10 +456,13 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
             v += __shfl_xor_sync(0xffffffffu, v, 2);
             r8[nt] = v;  // columns nt*8 + (0..7)
           }
-          const double r16a = r8[0] + r8[1], r16b = r8[2] + r8[3];
-          rsum[mt][h] = r16a + r16b;
+          // pairwise tree over the warp's NT column groups: r16[q] covers 16 columns
+          double r16[NT / 2 > 0 ? NT / 2 : 1];
+#pragma unroll
+          for (int q = 0; q < NT / 2; ++q) r16[q] = r8[2 * q] + r8[2 * q + 1];
+          double rw = NT == 4 ? r16[0] + r16[1] : r16[0];  // the warp's WTN columns
           const int64_t row = rbase + mt * 16 + h * 8 + g;
-          if (bs <= 32 && tig == 0 && row < args.M) {
+          if (tig == 0 && row < args.M) {
             if (bs == 8) {
 #pragma unroll
               for (int nt = 0; nt < NT; ++nt) {
@@ -456,40 +470,22 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
                 if (J < nJ) args.Rrow[row * nJ + J] = r8[nt];
               }
             } else if (bs == 16) {
-              const int64_t J0 = cbase / 16;
-              if (J0 < nJ) args.Rrow[row * nJ + J0] = r16a;
-              if (J0 + 1 < nJ) args.Rrow[row * nJ + J0 + 1] = r16b;
-            } else {
+#pragma unroll
+              for (int q = 0; q < NT / 2; ++q) {
+                const int64_t J = (cbase + q * 16) / 16;
+                if (J < nJ) args.Rrow[row * nJ + J] = r16[q];
+              }
+            } else if (bs < WTN) {  // bs = 32 inside a 32-column warp tile (NT == 4)
               const int64_t J = cbase / 32;
-              if (J < nJ) args.Rrow[row * nJ + J] = rsum[mt][h];
+              if (J < nJ) args.Rrow[row * nJ + J] = rw;
+            } else {  // block spans bs / WTN warp columns: part = which one
+              const int64_t J = cbase / bs;
+              const int part = (int)((cbase % bs) / WTN);
+              double *dst = part == 0 ? args.Rrow : args.Rrow2 + (int64_t)(part - 1) * args.M * nJ;
+              if (J < nJ) dst[row * nJ + J] = rw;
             }
           }
         }
-      if (bs == 64) {  // the whole tile is one block: each half-warp-grid writes its own
-        // partial (no inter-warp barrier in the epilogue); aabft_check adds the two halves in
-        // a fixed order (wm = 0 + wm = 1, wn = 0 + wn = 1)
-        const int64_t I = (int64_t)tl.m0 / 64, J = (int64_t)tl.n0 / 64;
-        double *rc = wm == 0 ? args.Rcol : args.Rcol2;
-        double *rr = wn == 0 ? args.Rrow : args.Rrow2;
-        if (g == 0) {
-#pragma unroll
-          for (int nt = 0; nt < NT; ++nt)
-#pragma unroll
-            for (int e = 0; e < 2; ++e) {
-              const int64_t c = cbase + nt * 8 + tig * 2 + e;
-              if (c < args.N) rc[I * args.N + c] = csum[nt][e];
-            }
-        }
-        if (tig == 0) {
-#pragma unroll
-          for (int mt = 0; mt < MT; ++mt)
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-              const int64_t r = rbase + mt * 16 + h * 8 + g;
-              if (r < args.M) rr[r * nJ + J] = rsum[mt][h];
-            }
-        }
-      }
     }
     double *out;
     int64_t ld, rows_valid, cols_valid;
@@ -562,13 +558,17 @@ static size_t red_off() {
   return r256z((size_t)kMaxCtas * ACC * THREADS * sizeof(double) + kMaxCtas * sizeof(int));
 }
 size_t gemm_f64_ws_bytes(const aabft_config *cfg) {
-  return red_off() + r256z((size_t)(cfg->M / cfg->bs) * cfg->N * 8) +
-         r256z((size_t)cfg->M * (cfg->N / cfg->bs) * 8) + 256;
+  return red_off() + r256z((size_t)(cfg->M / cfg->bs) * cfg->N * 8 * (COL_PARTS - 1)) +
+         r256z((size_t)cfg->M * (cfg->N / cfg->bs) * 8 * (ROW_PARTS - 1)) + 256;
+}
+int gemm_f64_fused_parts(int bs, int *row_parts) {
+  *row_parts = bs > WTN ? bs / WTN : 1;
+  return bs > 32 ? bs / 32 : 1;
 }
 void gemm_f64_red_ptrs(const aabft_config *cfg, void *ws, double **rcol2, double **rrow2) {
   char *w = static_cast<char *>(ws) + red_off();
   *rcol2 = reinterpret_cast<double *>(w);
-  *rrow2 = reinterpret_cast<double *>(w + r256z((size_t)(cfg->M / cfg->bs) * cfg->N * 8));
+  *rrow2 = reinterpret_cast<double *>(w + r256z((size_t)(cfg->M / cfg->bs) * cfg->N * 8 * (COL_PARTS - 1)));
 }
 
 aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
