@@ -149,6 +149,10 @@ aabft_status aabft_encode(const aabft_config *cfg, const void *A, int64_t lda, c
     set_error("encode B: need ldb >= N, Bcs (ld_bcs >= N/bs), topB_val, topB_idx");
     return AABFT_EINVAL;
   }
+  if ((A && !pitch_ok(cfg, A, lda)) || (B && !pitch_ok(cfg, B, ldb))) {
+    set_error("encode: A/B must be 16-byte aligned with row pitches that are multiples of 16 bytes");
+    return AABFT_EINVAL;
+  }
   if (!ws || ws_bytes < aabft_workspace_bytes(cfg)) {
     set_error("workspace too small: need %zu bytes", aabft_workspace_bytes(cfg));
     return AABFT_EWORKSPACE;

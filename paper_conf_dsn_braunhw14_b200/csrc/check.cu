@@ -70,6 +70,14 @@ __device__ __forceinline__ double ratio_of(double d, double eps) {
   return a == 0.0 ? 0.0 : CUDART_INF;
 }
 
+// |d| / eps for the report (a diagnostic: single-precision division is enough, no DDIV)
+__device__ __forceinline__ double ratio_fast(double d, double eps) {
+  const double a = fabs(d);
+  if (a != a) return CUDART_INF;
+  if (eps > 0.0) return (double)__fdividef((float)a, (float)eps);
+  return a == 0.0 ? 0.0 : CUDART_INF;
+}
+
 // atomic max on non-negative doubles (bit pattern order == value order)
 __device__ __forceinline__ void atomic_max_nonneg(double *addr, double v) {
   atomicMax(reinterpret_cast<unsigned long long *>(addr),
@@ -232,67 +240,113 @@ __global__ void __launch_bounds__(kCheckThreads) check_kernel(CheckArgs a, Bound
 
 // --------------------------------------------------------------------------- fused check
 // The GEMM epilogue already produced the reference sums (Rcol, Rrow); compare them with the
-// carried checksums: 2*bs checks per block, no pass over C.
+// carried checksums: 2*bs checks per block, no pass over C.  One WARP per block (grid-stride),
+// warp-shuffle reductions for the verdict, and the counters aggregated per CTA so the device
+// counters see one atomic per CTA instead of one per block.
 template <typename T, int P>
-__global__ void __launch_bounds__(128) check_fused_kernel(CheckArgs a, BoundParams bp) {
-  __shared__ int s_cls[3], s_nr, s_nc, s_row, s_col;
-  __shared__ double s_ratio[4];
-  const int bs = a.bs, tid = threadIdx.x, lane = tid & 31;
+__global__ void __launch_bounds__(256) check_fused_kernel(CheckArgs a, BoundParams bp, int64_t nb) {
+  __shared__ unsigned long long s_n[8];
+  __shared__ unsigned long long s_mr;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tid < 8) s_n[tid] = 0ull;
+  if (tid == 8) s_mr = 0ull;
+  __syncthreads();
+  const int bs = a.bs;
   const int64_t nJ = a.N / bs;
-  const int64_t I = blockIdx.x / nJ, J = blockIdx.x % nJ;
-  if (tid < 3) s_cls[tid] = 0;
-  if (tid == 0) { s_nr = 0; s_nc = 0; s_row = -1; s_col = -1; }
-  __syncthreads();
-  int cls_local[3] = {0, 0, 0};
-  double rmax = 0.0;
-  for (int e = tid; e < 2 * bs; e += 128) {
-    double d;
-    Bound b;
-    if (e < bs) {  // column check j
-      const int64_t j = J * bs + e;
-      double ref = a.Rcol[I * a.N + j];
-      if (a.col_parts > 1) {  // complete the epilogue parts (and leave the full sum in Rcol)
-        ref = ref + a.Rcol2[I * a.N + j];
-        const_cast<double *>(a.Rcol)[I * a.N + j] = ref;
+  unsigned long long my_n[8] = {0, 0, 0, 0, 0, 0, 0, 0};  // lane 0 of each warp
+  double my_mr = 0.0;
+  const int nJ32 = (int)nJ;
+  for (int blk = blockIdx.x * 8 + warp; blk < (int)nb; blk += gridDim.x * 8) {
+    const int I32 = blk / nJ32, J32 = blk - (blk / nJ32) * nJ32;
+    const int64_t I = I32, J = J32;
+    // per-block base pointers (32-bit offsets inside the block)
+    const double *rcol = a.Rcol + I * a.N + J * bs;
+    const double *rcol2 = a.col_parts > 1 ? a.Rcol2 + I * a.N + J * bs : nullptr;
+    const T *ccol_p = static_cast<const T *>(a.Ccol) + I * a.ld_ccol + J * bs;
+    const double *rrow = a.Rrow + (I * bs) * nJ + J;
+    const T *crow_p = static_cast<const T *>(a.Crow) + (I * bs) * a.ld_crow + J;
+    const double *tva_c = a.tav + (a.M + I) * P;
+    const int *tia_c = a.tai + (a.M + I) * P;
+    const double *tvb_r = a.tbv + (a.N + J) * P;
+    const int *tib_r = a.tbi + (a.N + J) * P;
+    int cls[3] = {0, 0, 0}, nr = 0, nc = 0, crow = -1, ccol = -1;
+    double rmax = 0.0;
+    for (int e = lane; e < 2 * bs; e += 32) {
+      double d;
+      Bound b;
+      if (e < bs) {  // column check j
+        const int j = J32 * bs + e;
+        double ref = rcol[e];
+        if (rcol2) {  // complete the epilogue parts (and leave the full sum in Rcol)
+          ref = ref + rcol2[e];
+          const_cast<double *>(rcol)[e] = ref;
+        }
+        d = ref - (double)ccol_p[e];
+        b = bound_of(bp, y_bound<P>(tva_c, tia_c, a.tbv + (int64_t)j * P, a.tbi + (int64_t)j * P));
+        const int cl = classify(d, b);
+        cls[cl] += 1;
+        if (cl == 2) { nc += 1; ccol = (int)j; }
+      } else {  // row check i
+        const int ii = e - bs;
+        const int64_t i = I * bs + ii;
+        double ref = rrow[(int64_t)ii * nJ];
+        if (a.row_parts > 1) {
+          for (int q = 1; q < a.row_parts; ++q) ref = ref + a.Rrow2[(q - 1) * a.M * nJ + i * nJ + J];
+          const_cast<double *>(rrow)[(int64_t)ii * nJ] = ref;
+        }
+        d = ref - (double)crow_p[(int64_t)ii * a.ld_crow];
+        b = bound_of(bp, y_bound<P>(a.tav + i * P, a.tai + i * P, tvb_r, tib_r));
+        const int cl = classify(d, b);
+        cls[cl] += 1;
+        if (cl == 2) { nr += 1; crow = (int)i; }
       }
-      d = ref - (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
-      b = bound_of(bp, y_bound<P>(a.tav + (a.M + I) * P, a.tai + (a.M + I) * P, a.tbv + j * P,
-                                  a.tbi + j * P));
-      const int cl = classify(d, b);
-      cls_local[cl] += 1;
-      if (cl == 2) { atomicAdd(&s_nc, 1); s_col = (int)j; }
-    } else {  // row check i
-      const int64_t i = I * bs + (e - bs);
-      double ref = a.Rrow[i * nJ + J];
-      if (a.row_parts > 1) {
-        for (int q = 1; q < a.row_parts; ++q) ref = ref + a.Rrow2[(q - 1) * a.M * nJ + i * nJ + J];
-        const_cast<double *>(a.Rrow)[i * nJ + J] = ref;
-      }
-      d = ref - (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
-      b = bound_of(bp, y_bound<P>(a.tav + i * P, a.tai + i * P, a.tbv + (a.N + J) * P,
-                                  a.tbi + (a.N + J) * P));
-      const int cl = classify(d, b);
-      cls_local[cl] += 1;
-      if (cl == 2) { atomicAdd(&s_nr, 1); s_row = (int)i; }
+      rmax = fmax(rmax, ratio_fast(d, b.eps));
     }
-    rmax = fmax(rmax, ratio_of(d, b.eps));
+#pragma unroll
+    for (int m = 16; m >= 1; m >>= 1) {
+      cls[0] += __shfl_xor_sync(0xffffffffu, cls[0], m);
+      cls[1] += __shfl_xor_sync(0xffffffffu, cls[1], m);
+      cls[2] += __shfl_xor_sync(0xffffffffu, cls[2], m);
+      nr += __shfl_xor_sync(0xffffffffu, nr, m);
+      nc += __shfl_xor_sync(0xffffffffu, nc, m);
+      crow = max(crow, __shfl_xor_sync(0xffffffffu, crow, m));
+      ccol = max(ccol, __shfl_xor_sync(0xffffffffu, ccol, m));
+      rmax = fmax(rmax, __shfl_xor_sync(0xffffffffu, rmax, m));
+    }
+    if (lane == 0) {
+      uint8_t status;
+      if (nr == 0 && nc == 0) status = AABFT_BLK_CLEAN;
+      else if (nr == 1 && nc == 1) status = AABFT_BLK_SINGLE;
+      else if (nr == 0 || nc == 0) status = AABFT_BLK_CHECKSUM_ONLY;
+      else status = AABFT_BLK_UNCORRECTABLE;
+      aabft_block_report r;
+      r.status = status;
+      r.worst_class = (uint8_t)(cls[2] ? 2 : (cls[1] ? 1 : 0));
+      r.n_bad_rows = (uint16_t)min(nr, 65535);
+      r.n_bad_cols = (uint16_t)min(nc, 65535);
+      r.reserved = 0;
+      r.row = status == AABFT_BLK_SINGLE ? crow : -1;
+      r.col = status == AABFT_BLK_SINGLE ? ccol : -1;
+      r.max_ratio = (float)rmax;
+      a.rep[blk] = r;
+      my_n[0] += 1;
+      my_n[1] += status == AABFT_BLK_CLEAN;
+      my_n[3] += status == AABFT_BLK_CHECKSUM_ONLY;
+      my_n[4] += status == AABFT_BLK_UNCORRECTABLE;
+      my_n[5] += cls[0];
+      my_n[6] += cls[1];
+      my_n[7] += cls[2];
+      my_mr = fmax(my_mr, rmax);
+    }
   }
-#pragma unroll
-  for (int c = 0; c < 3; ++c) {
-    int v = cls_local[c];
-#pragma unroll
-    for (int m = 16; m >= 1; m >>= 1) v += __shfl_xor_sync(0xffffffffu, v, m);
-    if (lane == 0 && v) atomicAdd(&s_cls[c], v);
+  if (lane == 0) {
+    for (int c = 0; c < 8; ++c)
+      if (my_n[c]) atomicAdd(&s_n[c], my_n[c]);
+    if (my_mr > 0.0) atomicMax(&s_mr, (unsigned long long)__double_as_longlong(my_mr));
   }
-#pragma unroll
-  for (int m = 16; m >= 1; m >>= 1) rmax = fmax(rmax, __shfl_xor_sync(0xffffffffu, rmax, m));
-  if (lane == 0) s_ratio[tid >> 5] = rmax;
   __syncthreads();
-  if (tid == 0) {
-    const double br = fmax(fmax(s_ratio[0], s_ratio[1]), fmax(s_ratio[2], s_ratio[3]));
-    const int cls[3] = {s_cls[0], s_cls[1], s_cls[2]};
-    finish_block(a, blockIdx.x, s_nr, s_nc, s_row, s_col, cls, br);
-  }
+  if (tid < 8 && s_n[tid]) atomicAdd(reinterpret_cast<unsigned long long *>(a.cnt->n) + tid, s_n[tid]);
+  if (tid == 8 && s_mr) atomicMax(reinterpret_cast<unsigned long long *>(&a.cnt->max_ratio), s_mr);
 }
 
 // --------------------------------------------------------------------------- correct
@@ -365,7 +419,8 @@ aabft_status run_check(const aabft_config *cfg, const CheckArgs &a, BoundParams 
   }
   if (nb > 0) {
     if (a.Rcol && a.Rrow) {
-      check_fused_kernel<T, P><<<(unsigned)nb, 128, 0, st>>>(a, bp);
+      const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((nb + 7) / 8, 148 * 8));
+      check_fused_kernel<T, P><<<grid, 256, 0, st>>>(a, bp, nb);
     } else {
       kern<<<(unsigned)nb, kCheckThreads, smem, st>>>(a, bp);
     }
