@@ -146,6 +146,7 @@ typedef struct {
  *          ("errorVecAdd1" at k-tile granularity; products inside the DMMA unit
  *          are not addressable)
  *  site 2: add `add` to the stored result (magnitude sweep)
+ *  site 3: add `add` to the accumulator after the k-tile that contains k_step
  * Capacity: the FP64 kernel applies at most 64 faults per 64 x 64 tile of C / Ccol / Crow, the
  * FP32 kernel at most 256 per 128 x 128 tile (i.e. one per 8 x 8 block); extra faults in the
  * same tile are ignored. */
@@ -170,6 +171,14 @@ size_t aabft_workspace_bytes(const aabft_config *cfg);
 aabft_status aabft_encode(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
                           int64_t ldb, const aabft_encoded *out, void *ws, size_t ws_bytes,
                           void *stream);
+
+/* Bound of arbitrary elements of C_fc (§IV-E last paragraph: "for each element c_ij of
+ * the full-checksum result matrix C_fc, this upper bound gives an expectation value and a
+ * variance"): for n DEVICE (row, col) pairs in C_fc coordinates (row >= M: checksum row of A,
+ * col >= N: checksum column of B) writes sigma and eps (double, device, n each). */
+aabft_status aabft_bound_elements(const aabft_config *cfg, const aabft_encoded *enc,
+                                  const int64_t *rows, const int64_t *cols, int64_t n,
+                                  double *sig, double *eps, void *stream);
 
 /* Bound alone (§IV-E): eps for every carried checksum element.
  * eps_col: (M/bs) x N dense, eps_row: M x (N/bs) dense (either may be NULL); sig_* likewise.

@@ -186,6 +186,7 @@ void oracle_gemm(int dtype, int fma_model, int64_t M, int64_t N, int64_t K, cons
  * site 0: XOR xor_mask into the bits of the final value ("errorVecAdd2")
  * site 1: XOR xor_mask into the partial sum right after step k_step ("errorVecAdd1")
  * site 2: add `add` to the final value (additive magnitude fault; R23)
+ * site 3: add `add` to the partial sum right after step k_step (additive accumulator fault)
  * The row a (len K, stride 1) and column b (len K, stride ldb) are passed directly. */
 static uint64_t bits_of(double x) { uint64_t u; memcpy(&u, &x, 8); return u; }
 static double of_bits(uint64_t u) { double x; memcpy(&x, &u, 8); return x; }
@@ -200,6 +201,7 @@ double oracle_dot_fault(int dtype, int fma_model, int64_t K, const void *a, cons
     for (int64_t k = 0; k < K; ++k) {
       c = fma_model ? fma(x[k], y[k * ldb], c) : c + x[k] * y[k * ldb];
       if (site == 1 && k == k_step) c = of_bits(bits_of(c) ^ xor_mask);
+      if (site == 3 && k == k_step) c = c + add;
     }
     if (site == 0) c = of_bits(bits_of(c) ^ xor_mask);
     if (site == 2) c = c + add;
@@ -210,6 +212,7 @@ double oracle_dot_fault(int dtype, int fma_model, int64_t K, const void *a, cons
     for (int64_t k = 0; k < K; ++k) {
       c = fma_model ? fmaf(x[k], y[k * ldb], c) : c + x[k] * y[k * ldb];
       if (site == 1 && k == k_step) c = of_bits_f(bits_of_f(c) ^ (uint32_t)xor_mask);
+      if (site == 3 && k == k_step) c = (float)((double)c + add);
     }
     if (site == 0) c = of_bits_f(bits_of_f(c) ^ (uint32_t)xor_mask);
     if (site == 2) c = (float)((double)c + add);

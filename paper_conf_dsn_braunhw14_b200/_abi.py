@@ -19,7 +19,8 @@ BLK_CLEAN, BLK_CORRECTED, BLK_CHECKSUM_ONLY, BLK_UNCORRECTABLE, BLK_SINGLE = 0, 
 STATUS_NAMES = {0: "CLEAN", 1: "CORRECTED", 2: "CHECKSUM_ONLY", 3: "UNCORRECTABLE", 4: "SINGLE"}
 COUNT_NAMES = ("blocks", "clean", "corrected", "checksum_only", "uncorrectable",
                "checks_rounding", "checks_tolerable", "checks_critical")
-EXPORTED = ("aabft_workspace_bytes", "aabft_encode", "aabft_bound", "aabft_gemm",
+EXPORTED = ("aabft_workspace_bytes", "aabft_encode", "aabft_bound", "aabft_bound_elements",
+            "aabft_gemm",
             "aabft_gemm_plain", "aabft_check", "aabft_correct", "aabft_host_arena_bytes",
             "aabft_protected_gemm_host", "aabft_status_str", "aabft_last_error",
             "aabft_version", "aabft_launch_count")
@@ -93,6 +94,7 @@ def lib():
         L.aabft_host_arena_bytes.restype = sz
         L.aabft_encode.argtypes = [pc, vp, i64, vp, i64, C.POINTER(Encoded), vp, sz, vp]
         L.aabft_bound.argtypes = [pc, C.POINTER(Encoded), vp, vp, vp, vp, vp]
+        L.aabft_bound_elements.argtypes = [pc, C.POINTER(Encoded), vp, vp, i64, vp, vp, vp]
         L.aabft_gemm.argtypes = [pc, vp, i64, vp, i64, C.POINTER(Encoded), C.POINTER(Product), vp,
                                  i32, vp, sz, vp]
         L.aabft_gemm_plain.argtypes = [pc, vp, i64, vp, i64, vp, i64, vp, sz, vp]
@@ -104,7 +106,7 @@ def lib():
         L.aabft_last_error.restype = C.c_char_p
         L.aabft_version.restype = C.c_char_p
         L.aabft_launch_count.restype = i64
-        for name in ("aabft_encode", "aabft_bound", "aabft_gemm", "aabft_gemm_plain",
+        for name in ("aabft_encode", "aabft_bound", "aabft_bound_elements", "aabft_gemm", "aabft_gemm_plain",
                      "aabft_check", "aabft_correct", "aabft_protected_gemm_host"):
             getattr(L, name).restype = C.c_int
         _lib = L

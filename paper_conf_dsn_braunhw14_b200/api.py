@@ -200,6 +200,18 @@ class ProtectedGemm:
                              _stream_ptr(stream)), "aabft_bound")
         return dict(eps_col=eps_col, sig_col=sig_col, eps_row=eps_row, sig_row=sig_row)
 
+    def bound_elements(self, rows, cols, stream=None):
+        """sigma, eps of arbitrary C_fc elements; rows/cols: int64 CUDA tensors."""
+        rows = rows.to(device=self.device, dtype=torch.int64).contiguous()
+        cols = cols.to(device=self.device, dtype=torch.int64).contiguous()
+        n = rows.numel()
+        sig = torch.empty(n, dtype=torch.float64, device=self.device)
+        eps = torch.empty(n, dtype=torch.float64, device=self.device)
+        ok(lib().aabft_bound_elements(C.byref(self.cfg), C.byref(self.enc), rows.data_ptr(),
+                                      cols.data_ptr(), n, sig.data_ptr(), eps.data_ptr(),
+                                      _stream_ptr(stream)), "aabft_bound_elements")
+        return sig, eps
+
     def run(self, A, B, *, faults=None, correct: bool = True, stream=None) -> Result:
         """encode -> gemm -> check -> correct, all enqueued on one stream."""
         self._check_operand(A, self.M, self.K, "A")

@@ -176,6 +176,25 @@ aabft_status aabft_bound(const aabft_config *cfg, const aabft_encoded *enc, doub
   AABFT_GUARD_END
 }
 
+aabft_status aabft_bound_elements(const aabft_config *cfg, const aabft_encoded *enc,
+                                  const int64_t *rows, const int64_t *cols, int64_t n,
+                                  double *sig, double *eps, void *stream) {
+  AABFT_GUARD_BEGIN
+  aabft_status s = validate(cfg);
+  if (s != AABFT_OK) return s;
+  if (!enc || !enc->topA_val || !enc->topA_idx || !enc->topB_val || !enc->topB_idx) {
+    set_error("bound_elements: top-p tables required");
+    return AABFT_EINVAL;
+  }
+  if (n < 0 || (n > 0 && (!rows || !cols || (!sig && !eps)))) {
+    set_error("bound_elements: rows, cols and sig or eps required");
+    return AABFT_EINVAL;
+  }
+  if ((s = device_ok()) != AABFT_OK) return s;
+  return launch_bound_elements(cfg, enc, rows, cols, n, sig, eps, (cudaStream_t)stream);
+  AABFT_GUARD_END
+}
+
 static aabft_status gemm_common(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
                                 int64_t ldb, const aabft_encoded *enc, const aabft_product *out,
                                 const aabft_fault *faults, int32_t nfaults, bool plain,

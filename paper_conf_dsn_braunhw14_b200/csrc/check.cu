@@ -110,6 +110,29 @@ __global__ void bound_kernel(int64_t M, int64_t N, int bs, BoundParams bp,
   }
 }
 
+// bound of arbitrary C_fc elements (row / col index straight into the top-p tables, whose
+// data vectors come first and checksum vectors after)
+template <int P>
+__global__ void bound_elements_kernel(int64_t M, int64_t N, int bs, BoundParams bp,
+                                      const double *__restrict__ tav, const int *__restrict__ tai,
+                                      const double *__restrict__ tbv, const int *__restrict__ tbi,
+                                      const int64_t *__restrict__ rows,
+                                      const int64_t *__restrict__ cols, int64_t n, double *sig,
+                                      double *eps) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < n;
+       e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = rows[e], c = cols[e];
+    double sg = CUDART_NAN, ep = CUDART_NAN;
+    if (r >= 0 && r < M + M / bs && c >= 0 && c < N + N / bs) {
+      const Bound b = bound_of(bp, y_bound<P>(tav + r * P, tai + r * P, tbv + c * P, tbi + c * P));
+      sg = b.sig;
+      ep = b.eps;
+    }
+    if (sig) sig[e] = sg;
+    if (eps) eps[e] = ep;
+  }
+}
+
 // --------------------------------------------------------------------------- check
 struct CheckArgs {
   int64_t M, N;
@@ -486,6 +509,23 @@ aabft_status launch_bound(const aabft_config *cfg, const aabft_encoded *enc, dou
                                            sig_col, eps_row, sig_row);
     next_launch();
     return check_launch("aabft_bound");
+  });
+  set_error("p out of range");
+  return AABFT_EINVAL;
+}
+
+aabft_status launch_bound_elements(const aabft_config *cfg, const aabft_encoded *enc,
+                                   const int64_t *rows, const int64_t *cols, int64_t n,
+                                   double *sig, double *eps, cudaStream_t st) {
+  const BoundParams bp = make_bound_params(cfg);
+  if (n <= 0) return AABFT_OK;
+  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, 148 * 16);
+  AABFT_P_SWITCH(cfg->p, {
+    bound_elements_kernel<PP><<<grid, 256, 0, st>>>(cfg->M, cfg->N, cfg->bs, bp, enc->topA_val,
+                                                    enc->topA_idx, enc->topB_val, enc->topB_idx,
+                                                    rows, cols, n, sig, eps);
+    next_launch();
+    return check_launch("aabft_bound_elements");
   });
   set_error("p out of range");
   return AABFT_EINVAL;

@@ -193,14 +193,16 @@ __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs ar
     if (nf > 0) {
       for (int f = 0; f < nf; ++f) {
         const aabft_fault ft = s_f[f];
-        if (ft.site != 1 || ft.k_step / BK != kt) continue;
+        if ((ft.site != 1 && ft.site != 3) || ft.k_step / BK != kt) continue;
 #pragma unroll
         for (int i = 0; i < 8; ++i)
 #pragma unroll
           for (int j = 0; j < 8; ++j) {
             const int r = (i < 4 ? ty * 4 + i : 64 + ty * 4 + i - 4);
             const int c = (j < 4 ? tx * 4 + j : HN + tx * 4 + j - 4);
-            if (r == ft.row && c == ft.col) ACC(i, j) = xor_bits(ACC(i, j), ft.xor_mask);
+            if (r == ft.row && c == ft.col)
+              ACC(i, j) = ft.site == 1 ? xor_bits(ACC(i, j), ft.xor_mask)
+                                       : (float)((double)ACC(i, j) + ft.add);
           }
       }
     }
@@ -210,7 +212,7 @@ __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs ar
   if (nf > 0) {
     for (int f = 0; f < nf; ++f) {
       const aabft_fault ft = s_f[f];
-      if (ft.site == 1) continue;
+      if (ft.site == 1 || ft.site == 3) continue;
 #pragma unroll
       for (int i = 0; i < 8; ++i)
 #pragma unroll

@@ -324,7 +324,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
       if (nf > 0) {  // Alg 3 errorVecAdd1 at k-tile granularity
         for (int f = 0; f < nf; ++f) {
           const aabft_fault ft = s_f[f];
-          if (ft.site != 1 || ft.k_step / BK != kt) continue;
+          if ((ft.site != 1 && ft.site != 3) || ft.k_step / BK != kt) continue;
 #pragma unroll
           for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
@@ -333,7 +333,9 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
               for (int q = 0; q < 4; ++q) {
                 const int64_t r = rbase + mt * 16 + g + (q >> 1) * 8;
                 const int64_t c = cbase + nt * 8 + tig * 2 + (q & 1);
-                if (r == ft.row && c == ft.col) acc[mt][nt][q] = xor_bits(acc[mt][nt][q], ft.xor_mask);
+                if (r == ft.row && c == ft.col)
+                  acc[mt][nt][q] = ft.site == 1 ? xor_bits(acc[mt][nt][q], ft.xor_mask)
+                                                : acc[mt][nt][q] + ft.add;
               }
         }
       }
@@ -380,7 +382,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
     if (nf > 0) {
       for (int f = 0; f < nf; ++f) {
         const aabft_fault ft = s_f[f];
-        if (ft.site == 1) continue;
+        if (ft.site == 1 || ft.site == 3) continue;
 #pragma unroll
         for (int mt = 0; mt < MT; ++mt)
 #pragma unroll

@@ -411,3 +411,43 @@ def test_fused_reference_sums(P, orc, bs):
     assert np.max(np.abs(host(plan.Rcol) - Rcol)) <= 1e-14 * scale
     assert np.max(np.abs(host(plan.Rrow) - Rrow)) <= 1e-14 * scale
     assert res.counts()["checks_critical"] == 0
+
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_bound_elements_bit_exact(P, orc, dtype):
+    """aabft_bound_elements: sigma/eps of arbitrary C_fc elements (data and checksum) == oracle."""
+    M, N, K, bs, p = 128, 192, 211, 32, 3
+    A = gen("wide", M, K, 41, 0, dtype)
+    B = gen("uniform", K, N, 41, 1, dtype)
+    plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p)
+    plan.encode(to_dev(A), to_dev(B))
+    rng = np.random.default_rng(3)
+    rows = rng.integers(0, M + M // bs, 200)
+    cols = rng.integers(0, N + N // bs, 200)
+    sig, eps = plan.bound_elements(torch.from_numpy(rows), torch.from_numpy(cols))
+    torch.cuda.synchronize()
+    enc = orc.encode(A, B, bs, p)
+    (av, ai), (bv, bi) = enc["topA"], enc["topB"]
+    for n, (r, c) in enumerate(zip(rows, cols)):
+        y = orc.y_of(av[r], ai[r], bv[c], bi[c])
+        s_o, e_o = orc.bound(K, y, t=orc.default_t(dtype))
+        assert host(sig)[n] == s_o and host(eps)[n] == e_o
+
+
+def test_accumulator_additive_fault_site3(P, orc):
+    """site 3: additive fault into the accumulator mid-k (magnitude-sweep site of SURVEY §8(d))."""
+    M, N, K, bs, p = 256, 256, 512, 64, 2
+    A = gen("uniform", M, K, 42, 0)
+    B = gen("uniform", K, N, 42, 1)
+    plan = P.ProtectedGemm(M, N, K, dtype=torch.float64, bs=bs, p=p)
+    dA, dB = to_dev(A), to_dev(B)
+    clean = host(plan.run(dA, dB).C).copy()
+    faults = [dict(row=3, col=4, site=3, k_step=K // 2, add=1e-3),
+              dict(row=100, col=200, site=3, k_step=7, add=-0.5)]
+    res = plan.run(dA, dB, faults=faults, correct=False)
+    torch.cuda.synchronize()
+    C1 = host(res.C)
+    assert abs((C1[3, 4] - clean[3, 4]) - 1e-3) < 1e-12
+    assert abs((C1[100, 200] - clean[100, 200]) + 0.5) < 1e-12
+    rep = res.reports()
+    assert rep["status"][0, 0] == 4 and rep["status"][1, 3] == 4   # located (SINGLE)
