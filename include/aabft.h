@@ -213,6 +213,17 @@ aabft_status aabft_correct(const aabft_config *cfg, const aabft_encoded *enc,
                            const aabft_product *prod, aabft_block_report *reports,
                            aabft_counts *counts, void *stream);
 
+/* Bound-quality study (NEXT-1; §VI-B, Tables II/III): the signed rounding error of
+ * every carried checksum, err = carried - exact, where the exact inner product of the checksum
+ * vectors (Acs[I] . B[:, j], A[i] . Bcs[:, J]) is formed in double-double on the GPU (Dot2:
+ * FMA TwoProd + compensated TwoSum; the paper used GMP on the host).  err_col:
+ * (M/bs) x N, err_row: M x (N/bs), dense doubles.  Needs the outputs of aabft_encode and
+ * aabft_gemm.  A diagnostic, not part of the protected path. */
+aabft_status aabft_checksum_errors(const aabft_config *cfg, const void *A, int64_t lda,
+                                   const void *B, int64_t ldb, const aabft_encoded *enc,
+                                   const aabft_product *prod, double *err_col, double *err_row,
+                                   void *stream);
+
 /* All four steps on HOST buffers (end-to-end entry point): copies A_host (M x K, dense) and
  * B_host (K x N, dense) into `arena` (device, >= aabft_host_arena_bytes), runs encode, gemm,
  * check, correct, and copies C (M x N dense) into C_host and the counts into counts_host.

@@ -23,7 +23,7 @@ EXPORTED = ("aabft_workspace_bytes", "aabft_encode", "aabft_bound", "aabft_bound
             "aabft_gemm",
             "aabft_gemm_plain", "aabft_check", "aabft_correct", "aabft_host_arena_bytes",
             "aabft_protected_gemm_host", "aabft_status_str", "aabft_last_error",
-            "aabft_version", "aabft_launch_count")
+            "aabft_version", "aabft_launch_count", "aabft_checksum_errors")
 
 
 class Config(C.Structure):
@@ -95,6 +95,8 @@ def lib():
         L.aabft_encode.argtypes = [pc, vp, i64, vp, i64, C.POINTER(Encoded), vp, sz, vp]
         L.aabft_bound.argtypes = [pc, C.POINTER(Encoded), vp, vp, vp, vp, vp]
         L.aabft_bound_elements.argtypes = [pc, C.POINTER(Encoded), vp, vp, i64, vp, vp, vp]
+        L.aabft_checksum_errors.argtypes = [pc, vp, i64, vp, i64, C.POINTER(Encoded),
+                                            C.POINTER(Product), vp, vp, vp]
         L.aabft_gemm.argtypes = [pc, vp, i64, vp, i64, C.POINTER(Encoded), C.POINTER(Product), vp,
                                  i32, vp, sz, vp]
         L.aabft_gemm_plain.argtypes = [pc, vp, i64, vp, i64, vp, i64, vp, sz, vp]
@@ -106,7 +108,8 @@ def lib():
         L.aabft_last_error.restype = C.c_char_p
         L.aabft_version.restype = C.c_char_p
         L.aabft_launch_count.restype = i64
-        for name in ("aabft_encode", "aabft_bound", "aabft_bound_elements", "aabft_gemm", "aabft_gemm_plain",
+        for name in ("aabft_encode", "aabft_bound", "aabft_bound_elements", "aabft_checksum_errors",
+                     "aabft_gemm", "aabft_gemm_plain",
                      "aabft_check", "aabft_correct", "aabft_protected_gemm_host"):
             getattr(L, name).restype = C.c_int
         _lib = L

@@ -212,6 +212,17 @@ class ProtectedGemm:
                                       _stream_ptr(stream)), "aabft_bound_elements")
         return sig, eps
 
+    def checksum_errors(self, A, B, stream=None):
+        """carried - exact (double-double) for every carried checksum (NEXT-1, Tables II/III)."""
+        nI, nJ = self.M // self.bs, self.N // self.bs
+        err_col = torch.empty(nI, self.N, dtype=torch.float64, device=self.device)
+        err_row = torch.empty(self.M, nJ, dtype=torch.float64, device=self.device)
+        ok(lib().aabft_checksum_errors(C.byref(self.cfg), A.data_ptr(), A.stride(0), B.data_ptr(),
+                                       B.stride(0), C.byref(self.enc), C.byref(self.prod),
+                                       err_col.data_ptr(), err_row.data_ptr(), _stream_ptr(stream)),
+           "aabft_checksum_errors")
+        return err_col, err_row
+
     def run(self, A, B, *, faults=None, correct: bool = True, stream=None) -> Result:
         """encode -> gemm -> check -> correct, all enqueued on one stream."""
         self._check_operand(A, self.M, self.K, "A")

@@ -195,6 +195,23 @@ aabft_status aabft_bound_elements(const aabft_config *cfg, const aabft_encoded *
   AABFT_GUARD_END
 }
 
+aabft_status aabft_checksum_errors(const aabft_config *cfg, const void *A, int64_t lda,
+                                   const void *B, int64_t ldb, const aabft_encoded *enc,
+                                   const aabft_product *prod, double *err_col, double *err_row,
+                                   void *stream) {
+  AABFT_GUARD_BEGIN
+  aabft_status s = validate(cfg);
+  if (s != AABFT_OK) return s;
+  if (!A || !B || !enc || !enc->Acs || !enc->Bcs || !prod || !prod->Ccol || !prod->Crow ||
+      !err_col || !err_row || lda < cfg->K || ldb < cfg->N) {
+    set_error("checksum_errors: A, B, Acs, Bcs, Ccol, Crow, err_col, err_row required");
+    return AABFT_EINVAL;
+  }
+  if ((s = device_ok()) != AABFT_OK) return s;
+  return launch_checksum_errors(cfg, A, lda, B, ldb, enc, prod, err_col, err_row, (cudaStream_t)stream);
+  AABFT_GUARD_END
+}
+
 static aabft_status gemm_common(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
                                 int64_t ldb, const aabft_encoded *enc, const aabft_product *out,
                                 const aabft_fault *faults, int32_t nfaults, bool plain,

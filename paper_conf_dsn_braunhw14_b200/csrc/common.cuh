@@ -59,6 +59,10 @@ aabft_status launch_gemm_f32(const aabft_config *cfg, const void *A, int64_t lda
 aabft_status launch_bound_elements(const aabft_config *cfg, const aabft_encoded *enc,
                                    const int64_t *rows, const int64_t *cols, int64_t n,
                                    double *sig, double *eps, cudaStream_t st);
+aabft_status launch_checksum_errors(const aabft_config *cfg, const void *A, int64_t lda,
+                                    const void *B, int64_t ldb, const aabft_encoded *enc,
+                                    const aabft_product *prod, double *err_col, double *err_row,
+                                    cudaStream_t st);
 aabft_status launch_check(const aabft_config *cfg, const aabft_encoded *enc,
                           const aabft_product *prod, aabft_block_report *rep,
                           aabft_counts *cnt, void *gemm_ws, cudaStream_t st);

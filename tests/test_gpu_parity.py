@@ -451,3 +451,49 @@ def test_accumulator_additive_fault_site3(P, orc):
     assert abs((C1[100, 200] - clean[100, 200]) + 0.5) < 1e-12
     rep = res.reports()
     assert rep["status"][0, 0] == 4 and rep["status"][1, 3] == 4   # located (SINGLE)
+
+
+def test_checksum_errors_double_double(P, orc):
+    """NEXT-1 diagnostic: carried - exact checksum error with the exact inner product formed in
+    double-double on the GPU, against exact rational arithmetic (fractions) on sampled
+    elements; Dot2's own error (~2^-104 sum|terms|) is far below the tolerance."""
+    from fractions import Fraction
+    M, N, K, bs = 128, 128, 300, 32
+    A = gen("uniform", M, K, 51, 0)
+    B = gen("uniform", K, N, 51, 1)
+    plan = P.ProtectedGemm(M, N, K, dtype=torch.float64, bs=bs, p=2)
+    dA, dB = to_dev(A), to_dev(B)
+    res = plan.run(dA, dB)
+    ec, er = plan.checksum_errors(dA, dB)
+    torch.cuda.synchronize()
+    Acs, Bcs, Ccol, Crow = host(plan.Acs), host(plan.Bcs), host(res.Ccol), host(res.Crow)
+    ec, er = host(ec), host(er)
+    rng = np.random.default_rng(5)
+    for _ in range(24):
+        I, j = int(rng.integers(M // bs)), int(rng.integers(N))
+        exact = sum(Fraction(float(Acs[I, k])) * Fraction(float(B[k, j])) for k in range(K))
+        ref = float(Fraction(float(Ccol[I, j])) - exact)
+        assert abs(ec[I, j] - ref) <= 1e-28 + 1e-12 * abs(ref)
+        i, J = int(rng.integers(M)), int(rng.integers(N // bs))
+        exact = sum(Fraction(float(A[i, k])) * Fraction(float(Bcs[k, J])) for k in range(K))
+        ref = float(Fraction(float(Crow[i, J])) - exact)
+        assert abs(er[i, J] - ref) <= 1e-28 + 1e-12 * abs(ref)
+    assert np.abs(ec).max() > 0  # the GEMM does round
+
+
+@pytest.mark.parametrize("n", [512, 1024, 2048, 4096])
+@pytest.mark.parametrize("table", ["table2_uniform1.json", "table3_uniform100.json"])
+def test_gpu_bound_column_tables(P, orc, n, table):
+    """Published-number pin of the GPU encode + bound path at full size: mean eps over all
+    carried checksum elements (BS 32, p 2, 3 sigma, t 52) within 5% of Table II / III."""
+    import json, os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", table)))
+    A = gen(g["recipe"], n, n, 1, 0)
+    B = gen(g["recipe"], n, n, 2, 1)
+    plan = P.ProtectedGemm(n, n, n, dtype=torch.float64, bs=32, p=2)
+    plan.encode(to_dev(A), to_dev(B))
+    b = plan.bound()
+    torch.cuda.synchronize()
+    m = float(torch.cat([b["eps_col"].ravel(), b["eps_row"].ravel()]).mean())
+    paper = g["rows"][str(n)]["avg_aabft"]
+    assert 0.95 * paper <= m <= 1.05 * paper, (m, paper)
