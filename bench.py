@@ -170,7 +170,8 @@ def run_reference(args, wl):
     if rank != 0:
         return
     nthreads = os.cpu_count() or 1
-    rows = cpu_rows_for(wl, 8.0, nthreads)
+    # each step ~2 s of oracle work so that --steps K --warmup W ends within a few minutes
+    rows = cpu_rows_for(wl, 2.0, nthreads)
     for _ in range(args.warmup):
         oracle_sample(dict(wl, N=min(wl["N"], 256)), wl["bs"], nthreads)
     times, flops = [], 0.0
@@ -206,11 +207,17 @@ def main():
     import torch.distributed as dist
 
     rank, world, local = dist_env()
-    if world > 1:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    # one process per GPU; AABFT_DIST_BACKEND=gloo lets the multi-rank path be exercised with
+    # several ranks sharing one GPU (tests on a 1-GPU box), NCCL otherwise
+    backend = os.environ.get("AABFT_DIST_BACKEND", "nccl")
+    local = local % max(1, torch.cuda.device_count())
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
+    if world > 1:
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
 
     from paper_conf_dsn_braunhw14_b200 import _abi, api
 
