@@ -18,7 +18,10 @@
  * Pins (tests/test_oracle_*.py): closed forms of Eq 28 / P:L287, integer-exact checksum
  * identities (Eq 5), brute-force top-p and y invariants (§IV-E), the Table II/III
  * "AVG. A-ABFT" and "AVG. Rnd. Error" columns, brute-force single-fault
- * locate/correct on tiny integer inputs.  No function here is "parity unpinned".
+ * locate/correct on tiny integer inputs; the NEXT-3 comparators (external-eps check/correct,
+ * SEA-ABFT bound O11) and the Alg 3 product site (site 4) in tests/test_oracle_comparators.py,
+ * the SEA bound against Table II/III "AVG. SEA-ABFT".  No function here is
+ * "parity unpinned".
  */
 #include <math.h>
 #include <pthread.h>
@@ -187,6 +190,9 @@ void oracle_gemm(int dtype, int fma_model, int64_t M, int64_t N, int64_t K, cons
  * site 1: XOR xor_mask into the partial sum right after step k_step ("errorVecAdd1")
  * site 2: add `add` to the final value (additive magnitude fault; R23)
  * site 3: add `add` to the partial sum right after step k_step (additive accumulator fault)
+ * site 4: "errorVecMul" (Alg 3 inner loop: accum += (rA*rB) XOR errorVecMult):
+ *         at step k_step the product is rounded on its own, XOR-ed with xor_mask and then
+ *         added (c = c + (fl(a_k*b_k) ^ mask)); every other step as fma_model says
  * The row a (len K, stride 1) and column b (len K, stride ldb) are passed directly. */
 static uint64_t bits_of(double x) { uint64_t u; memcpy(&u, &x, 8); return u; }
 static double of_bits(uint64_t u) { double x; memcpy(&x, &u, 8); return x; }
@@ -199,7 +205,12 @@ double oracle_dot_fault(int dtype, int fma_model, int64_t K, const void *a, cons
     const double *x = (const double *)a, *y = (const double *)b;
     double c = 0.0;
     for (int64_t k = 0; k < K; ++k) {
-      c = fma_model ? fma(x[k], y[k * ldb], c) : c + x[k] * y[k * ldb];
+      if (site == 4 && k == k_step) {
+        double prod = x[k] * y[k * ldb];
+        c = c + of_bits(bits_of(prod) ^ xor_mask);
+      } else {
+        c = fma_model ? fma(x[k], y[k * ldb], c) : c + x[k] * y[k * ldb];
+      }
       if (site == 1 && k == k_step) c = of_bits(bits_of(c) ^ xor_mask);
       if (site == 3 && k == k_step) c = c + add;
     }
@@ -210,7 +221,12 @@ double oracle_dot_fault(int dtype, int fma_model, int64_t K, const void *a, cons
     const float *x = (const float *)a, *y = (const float *)b;
     float c = 0.0f;
     for (int64_t k = 0; k < K; ++k) {
-      c = fma_model ? fmaf(x[k], y[k * ldb], c) : c + x[k] * y[k * ldb];
+      if (site == 4 && k == k_step) {
+        float prod = x[k] * y[k * ldb];
+        c = c + of_bits_f(bits_of_f(prod) ^ (uint32_t)xor_mask);
+      } else {
+        c = fma_model ? fmaf(x[k], y[k * ldb], c) : c + x[k] * y[k * ldb];
+      }
       if (site == 1 && k == k_step) c = of_bits_f(bits_of_f(c) ^ (uint32_t)xor_mask);
       if (site == 3 && k == k_step) c = (float)((double)c + add);
     }
@@ -336,13 +352,53 @@ static double ratio_of(double d, double eps) {
   return a == 0.0 ? 0.0 : INFINITY;
 }
 
-void oracle_check(int dtype, int64_t M, int64_t N, int64_t K, int bs, int p, double omega, int t,
-                  int fma_model, const void *C, int64_t ldc, const void *Ccol, int64_t ld_ccol,
-                  const void *Crow, int64_t ld_crow, const double *topA_val,
-                  const int32_t *topA_idx, const double *topB_val, const int32_t *topB_idx,
-                  int32_t *rep_status, int32_t *rep_worst, int32_t *rep_nrows,
-                  int32_t *rep_ncols, int32_t *rep_row, int32_t *rep_col, double *rep_ratio,
-                  int64_t *counts, double *max_ratio, double *d_col, double *d_row) {
+/* Where eps (and sigma) of a carried checksum come from.  A-ABFT (the method): the bound of
+ * §IV-E from the top-p tables.  External (NEXT-3 comparators, reading R26): a caller-given
+ * eps per checksum (eps_col / eps_row, e.g. the SEA-ABFT bound) or, when those are NULL, one
+ * fixed eps for every check ("ABFT with manually set error bounds", Table I);
+ * external bounds carry no sigma, so sigma = eps (classes ROUNDING / CRITICAL only). */
+typedef struct {
+  int external;
+  int64_t M, N, K;
+  int bs, p, t, fma_model;
+  double omega;
+  const double *topA_val, *topB_val;
+  const int32_t *topA_idx, *topB_idx;
+  const double *eps_col, *eps_row;
+  double eps_fixed;
+} eps_source;
+
+static void col_bound(const eps_source *s, int64_t I, int64_t j, double *sg, double *e) {
+  if (s->external) {
+    *e = s->eps_col ? s->eps_col[I * s->N + j] : s->eps_fixed;
+    *sg = *e;
+    return;
+  }
+  int p = s->p;
+  double y = oracle_y(p, s->topA_val + (s->M + I) * p, s->topA_idx + (s->M + I) * p,
+                      s->topB_val + j * p, s->topB_idx + j * p);
+  oracle_bound(s->K, s->fma_model, s->t, s->omega, y, sg, e);
+}
+
+static void row_bound(const eps_source *s, int64_t i, int64_t J, double *sg, double *e) {
+  if (s->external) {
+    *e = s->eps_row ? s->eps_row[i * (s->N / s->bs) + J] : s->eps_fixed;
+    *sg = *e;
+    return;
+  }
+  int p = s->p;
+  double y = oracle_y(p, s->topA_val + i * p, s->topA_idx + i * p, s->topB_val + (s->N + J) * p,
+                      s->topB_idx + (s->N + J) * p);
+  oracle_bound(s->K, s->fma_model, s->t, s->omega, y, sg, e);
+}
+
+static void check_core(int dtype, const eps_source *src, const void *C, int64_t ldc,
+                       const void *Ccol, int64_t ld_ccol, const void *Crow, int64_t ld_crow,
+                       int32_t *rep_status, int32_t *rep_worst, int32_t *rep_nrows,
+                       int32_t *rep_ncols, int32_t *rep_row, int32_t *rep_col, double *rep_ratio,
+                       int64_t *counts, double *max_ratio, double *d_col, double *d_row) {
+  int64_t M = src->M, N = src->N;
+  int bs = src->bs;
   int64_t nI = M / bs, nJ = N / bs;
   for (int c = 0; c < 8; ++c) counts[c] = 0;
   *max_ratio = 0.0;
@@ -356,10 +412,8 @@ void oracle_check(int dtype, int64_t M, int64_t N, int64_t K, int bs, int p, dou
         double ref = 0.0;
         for (int64_t i = I * bs; i < I * bs + bs; ++i) ref = ref + ld(dtype, C, i * ldc + j);
         double d = ref - ld(dtype, Ccol, I * ld_ccol + j);
-        double y = oracle_y(p, topA_val + (M + I) * p, topA_idx + (M + I) * p,
-                            topB_val + j * p, topB_idx + j * p);
         double sg, e;
-        oracle_bound(K, fma_model, t, omega, y, &sg, &e);
+        col_bound(src, I, j, &sg, &e);
         int cl = classify(d, sg, e);
         counts[5 + cl] += 1;
         if (cl > worst) worst = cl;
@@ -373,10 +427,8 @@ void oracle_check(int dtype, int64_t M, int64_t N, int64_t K, int bs, int p, dou
         double ref = 0.0;
         for (int64_t j = J * bs; j < J * bs + bs; ++j) ref = ref + ld(dtype, C, i * ldc + j);
         double d = ref - ld(dtype, Crow, i * ld_crow + J);
-        double y = oracle_y(p, topA_val + i * p, topA_idx + i * p, topB_val + (N + J) * p,
-                            topB_idx + (N + J) * p);
         double sg, e;
-        oracle_bound(K, fma_model, t, omega, y, &sg, &e);
+        row_bound(src, i, J, &sg, &e);
         int cl = classify(d, sg, e);
         counts[5 + cl] += 1;
         if (cl > worst) worst = cl;
@@ -405,18 +457,46 @@ void oracle_check(int dtype, int64_t M, int64_t N, int64_t K, int bs, int p, dou
     }
 }
 
+void oracle_check(int dtype, int64_t M, int64_t N, int64_t K, int bs, int p, double omega, int t,
+                  int fma_model, const void *C, int64_t ldc, const void *Ccol, int64_t ld_ccol,
+                  const void *Crow, int64_t ld_crow, const double *topA_val,
+                  const int32_t *topA_idx, const double *topB_val, const int32_t *topB_idx,
+                  int32_t *rep_status, int32_t *rep_worst, int32_t *rep_nrows,
+                  int32_t *rep_ncols, int32_t *rep_row, int32_t *rep_col, double *rep_ratio,
+                  int64_t *counts, double *max_ratio, double *d_col, double *d_row) {
+  eps_source src = {0, M, N, K, bs, p, t, fma_model, omega, topA_val, topB_val, topA_idx,
+                    topB_idx, NULL, NULL, 0.0};
+  check_core(dtype, &src, C, ldc, Ccol, ld_ccol, Crow, ld_crow, rep_status, rep_worst, rep_nrows,
+             rep_ncols, rep_row, rep_col, rep_ratio, counts, max_ratio, d_col, d_row);
+}
+
+/* The same check against an external eps (NEXT-3 comparators; reading R26): eps_col
+ * ((M/bs) x N) and eps_row (M x (N/bs)) or, when both are NULL, eps_fixed everywhere. */
+void oracle_check_ext(int dtype, int64_t M, int64_t N, int bs, const void *C, int64_t ldc,
+                      const void *Ccol, int64_t ld_ccol, const void *Crow, int64_t ld_crow,
+                      const double *eps_col, const double *eps_row, double eps_fixed,
+                      int32_t *rep_status, int32_t *rep_worst, int32_t *rep_nrows,
+                      int32_t *rep_ncols, int32_t *rep_row, int32_t *rep_col, double *rep_ratio,
+                      int64_t *counts, double *max_ratio, double *d_col, double *d_row) {
+  eps_source src = {1, M, N, 0, bs, 0, 0, 0, 0.0, NULL, NULL, NULL, NULL, eps_col, eps_row,
+                    eps_fixed};
+  check_core(dtype, &src, C, ldc, Ccol, ld_ccol, Crow, ld_crow, rep_status, rep_worst, rep_nrows,
+             rep_ncols, rep_row, rep_col, rep_ratio, counts, max_ratio, d_col, d_row);
+}
+
 /* O8 correction (reading R15, Huang-Abraham [10]; Alg 2 "start correction"):
  * for every SINGLE(4) block with located (i, j):
  *   C[i][j] <- Ccol[I][j] - sum_{i' in I, i' != i} C[i'][j]   (double, ascending i'; stored in w)
  * then re-check row i against Crow[i][J] with its own eps: CORRECTED(1) if |d| <= eps,
  * else UNCORRECTABLE(3).  Updates counts[2] / counts[4]. */
-void oracle_correct(int dtype, int64_t M, int64_t N, int64_t K, int bs, int p, double omega, int t,
-                    int fma_model, void *C, int64_t ldc, const void *Ccol, int64_t ld_ccol,
-                    const void *Crow, int64_t ld_crow, const double *topA_val,
-                    const int32_t *topA_idx, const double *topB_val, const int32_t *topB_idx,
-                    int32_t *rep_status, const int32_t *rep_row, const int32_t *rep_col,
-                    int64_t *counts) {
+static void correct_core(int dtype, const eps_source *src, void *C, int64_t ldc,
+                         const void *Ccol, int64_t ld_ccol, const void *Crow, int64_t ld_crow,
+                         int32_t *rep_status, const int32_t *rep_row, const int32_t *rep_col,
+                         int64_t *counts) {
+  int64_t M = src->M, N = src->N;
+  int bs = src->bs;
   int64_t nI = M / bs, nJ = N / bs;
+  (void)M;
   for (int64_t I = 0; I < nI; ++I)
     for (int64_t J = 0; J < nJ; ++J) {
       int64_t b = I * nJ + J;
@@ -430,13 +510,91 @@ void oracle_correct(int dtype, int64_t M, int64_t N, int64_t K, int bs, int p, d
       double ref = 0.0;
       for (int64_t jj = J * bs; jj < J * bs + bs; ++jj) ref = ref + ld(dtype, C, i * ldc + jj);
       double d = ref - ld(dtype, Crow, i * ld_crow + J);
-      double y = oracle_y(p, topA_val + i * p, topA_idx + i * p, topB_val + (N + J) * p,
-                          topB_idx + (N + J) * p);
       double sg, e;
-      oracle_bound(K, fma_model, t, omega, y, &sg, &e);
+      row_bound(src, i, J, &sg, &e);
       if (fabs(d) <= e) { rep_status[b] = 1; counts[2] += 1; }
       else { rep_status[b] = 3; counts[4] += 1; }
     }
 }
 
-/* SEA-ABFT bound is a comparison system (OUT of scope); not implemented. */
+void oracle_correct(int dtype, int64_t M, int64_t N, int64_t K, int bs, int p, double omega, int t,
+                    int fma_model, void *C, int64_t ldc, const void *Ccol, int64_t ld_ccol,
+                    const void *Crow, int64_t ld_crow, const double *topA_val,
+                    const int32_t *topA_idx, const double *topB_val, const int32_t *topB_idx,
+                    int32_t *rep_status, const int32_t *rep_row, const int32_t *rep_col,
+                    int64_t *counts) {
+  eps_source src = {0, M, N, K, bs, p, t, fma_model, omega, topA_val, topB_val, topA_idx,
+                    topB_idx, NULL, NULL, 0.0};
+  correct_core(dtype, &src, C, ldc, Ccol, ld_ccol, Crow, ld_crow, rep_status, rep_row, rep_col,
+               counts);
+}
+
+/* Correction with the external eps of oracle_check_ext (the re-verified row uses eps_row, or
+ * eps_fixed when eps_row is NULL). */
+void oracle_correct_ext(int dtype, int64_t M, int64_t N, int bs, void *C, int64_t ldc,
+                        const void *Ccol, int64_t ld_ccol, const void *Crow, int64_t ld_crow,
+                        const double *eps_row, double eps_fixed, int32_t *rep_status,
+                        const int32_t *rep_row, const int32_t *rep_col, int64_t *counts) {
+  eps_source src = {1, M, N, 0, bs, 0, 0, 0, 0.0, NULL, NULL, NULL, NULL, NULL, eps_row,
+                    eps_fixed};
+  correct_core(dtype, &src, C, ldc, Ccol, ld_ccol, Crow, ld_crow, rep_status, rep_row, rep_col,
+               counts);
+}
+
+/* ------------------------------------------------------------------------------------
+ * O11 SEA-ABFT bound (NEXT-3 comparator, reporting only).  §III, the simplified
+ * error analysis bound of ref [28] for the column checksum of an (m+1) x n column-checksum
+ * matrix A times a column b:
+ *   |c_{n+1} - c*_{n+1}| < ((n + 2m - 2) ||b||_2 sum_{i=1..m} ||a_i||_2
+ *                          + n ||a_{m+1}||_2 ||b||_2) eps_M,          eps_M = 2^-t
+ * Partitioned encoding: m = bs rows of block-row I, a_{m+1} = Acs[I] (the checksum
+ * row), b = column j of B, n = K.  A row checksum (i, J) is the transposed statement (A, b)
+ * -> (B^T, a_i): the BS columns b_j of block-column J play a_1..a_m, Bcs[:, J] plays a_{m+1}
+ * and row a_i of A plays b.  The corner (I, J) (reading R25, only for the Table II/III
+ * average): a_{m+1} = Acs[I], b = Bcs[:, J].
+ * Norms: ||x||_2 = sqrt of the sequential ascending sum of x_k^2 in double.
+ * ------------------------------------------------------------------------------------ */
+static double norm_seq(int dtype, const void *X, int64_t off, int64_t len, int64_t stride) {
+  double s = 0.0;
+  for (int64_t k = 0; k < len; ++k) {
+    double v = ld(dtype, X, off + k * stride);
+    s = s + v * v;
+  }
+  return sqrt(s);
+}
+
+/* ||row r||_2 of an R x L row-major matrix (ld) -> out[r] */
+void oracle_norms_rows(int dtype, int64_t R, int64_t L, const void *X, int64_t ldx, double *out) {
+  for (int64_t r = 0; r < R; ++r) out[r] = norm_seq(dtype, X, r * ldx, L, 1);
+}
+
+/* ||column c||_2 of an L x Cn row-major matrix (ld) -> out[c] */
+void oracle_norms_cols(int dtype, int64_t L, int64_t Cn, const void *X, int64_t ldx, double *out) {
+  for (int64_t c = 0; c < Cn; ++c) out[c] = norm_seq(dtype, X, c, L, ldx);
+}
+
+/* nA[M] row norms of A, nAcs[M/bs] of the checksum rows, nB[N] column norms of B, nBcs[N/bs]
+ * of the checksum columns.  Outputs eps_col (M/bs) x N, eps_row M x (N/bs), eps_corner
+ * (M/bs) x (N/bs) (any may be NULL).  Evaluation: ((n+2m-2) * ||b|| * S + n * ||a_{m+1}|| *
+ * ||b||) * 2^-t with S = sequential ascending sum of the m norms. */
+void oracle_sea_bounds(int64_t M, int64_t N, int64_t K, int bs, int t, const double *nA,
+                       const double *nAcs, const double *nB, const double *nBcs, double *eps_col,
+                       double *eps_row, double *eps_corner) {
+  int64_t nI = M / bs, nJ = N / bs;
+  double n = (double)K, c1 = (double)K + 2.0 * bs - 2.0;
+  for (int64_t I = 0; I < nI; ++I) {
+    double SA = 0.0;
+    for (int64_t i = I * bs; i < I * bs + bs; ++i) SA = SA + nA[i];
+    for (int64_t j = 0; j < N; ++j)
+      if (eps_col) eps_col[I * N + j] = ldexp(c1 * nB[j] * SA + n * nAcs[I] * nB[j], -t);
+    for (int64_t J = 0; J < nJ; ++J)
+      if (eps_corner) eps_corner[I * nJ + J] = ldexp(c1 * nBcs[J] * SA + n * nAcs[I] * nBcs[J], -t);
+  }
+  for (int64_t J = 0; J < nJ; ++J) {
+    double SB = 0.0;
+    for (int64_t j = J * bs; j < J * bs + bs; ++j) SB = SB + nB[j];
+    for (int64_t i = 0; i < M; ++i)
+      if (eps_row) eps_row[i * nJ + J] = ldexp(c1 * nA[i] * SB + n * nBcs[J] * nA[i], -t);
+  }
+}
+

@@ -57,6 +57,13 @@ def lib():
                                    vp, vp]
         L.oracle_correct.argtypes = [i32, i64, i64, i64, i32, i32, dbl, i32, i32, vp, i64, vp,
                                      i64, vp, i64, vp, vp, vp, vp, vp, vp, vp, vp]
+        L.oracle_check_ext.argtypes = [i32, i64, i64, i32, vp, i64, vp, i64, vp, i64, vp, vp, dbl,
+                                       vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, vp]
+        L.oracle_correct_ext.argtypes = [i32, i64, i64, i32, vp, i64, vp, i64, vp, i64, vp, dbl,
+                                         vp, vp, vp, vp]
+        L.oracle_norms_rows.argtypes = [i32, i64, i64, vp, i64, vp]
+        L.oracle_norms_cols.argtypes = [i32, i64, i64, vp, i64, vp]
+        L.oracle_sea_bounds.argtypes = [i64, i64, i64, i32, i32, vp, vp, vp, vp, vp, vp, vp]
         _lib = L
     return _lib
 
@@ -225,6 +232,71 @@ def correct(Cm, Ccol, Crow, K, bs, p, topA, topB, res: CheckResult, *, omega=3.0
     return res
 
 
+def check_ext(Cm, Ccol, Crow, bs, *, eps_col=None, eps_row=None, eps_fixed=0.0):
+    """O7 against an external eps (NEXT-3, reading R26): per-checksum eps arrays (e.g. SEA) or
+    one fixed eps for every check."""
+    Cm, Ccol, Crow = _c(Cm), _c(Ccol), _c(Crow)
+    M, N = Cm.shape
+    nb = (M // bs) * (N // bs)
+    ints = [np.zeros(nb, np.int32) for _ in range(6)]
+    ratio = np.zeros(nb)
+    counts = np.zeros(8, np.int64)
+    mr = np.zeros(1)
+    d_col = np.zeros((M // bs, N))
+    d_row = np.zeros((M, N // bs))
+    ec = None if eps_col is None else _c(np.asarray(eps_col, np.float64))
+    er = None if eps_row is None else _c(np.asarray(eps_row, np.float64))
+    lib().oracle_check_ext(_dt(Cm), M, N, bs, _p(Cm), N, _p(Ccol), N, _p(Crow), N // bs, _p(ec),
+                           _p(er), float(eps_fixed), *[_p(x) for x in ints], _p(ratio),
+                           _p(counts), _p(mr), _p(d_col), _p(d_row))
+    shp = (M // bs, N // bs)
+    return CheckResult(*(x.reshape(shp) for x in ints), ratio.reshape(shp), counts,
+                       float(mr[0]), d_col, d_row)
+
+
+def correct_ext(Cm, Ccol, Crow, bs, res: CheckResult, *, eps_row=None, eps_fixed=0.0):
+    assert Cm.flags.c_contiguous
+    M, N = Cm.shape
+    st = _c(res.status.reshape(-1)).copy()
+    er = None if eps_row is None else _c(np.asarray(eps_row, np.float64))
+    lib().oracle_correct_ext(_dt(Cm), M, N, bs, _p(Cm), N, _p(_c(Ccol)), N, _p(_c(Crow)), N // bs,
+                             _p(er), float(eps_fixed), _p(st), _p(_c(res.row.reshape(-1))),
+                             _p(_c(res.col.reshape(-1))), _p(res.counts))
+    res.status = st.reshape(res.status.shape)
+    return res
+
+
+def norms_rows(X):
+    X = _c(X)
+    R, L = X.shape
+    out = np.zeros(R)
+    lib().oracle_norms_rows(_dt(X), R, L, _p(X), L, _p(out))
+    return out
+
+
+def norms_cols(X):
+    X = _c(X)
+    L, Cn = X.shape
+    out = np.zeros(Cn)
+    lib().oracle_norms_cols(_dt(X), L, Cn, _p(X), Cn, _p(out))
+    return out
+
+
+def sea_bounds(A, B, Acs, Bcs, bs, *, t=None):
+    """O11 SEA-ABFT comparator bound (§III): eps_col, eps_row and the corner."""
+    M, K = A.shape
+    N = B.shape[1]
+    t = default_t(A.dtype) if t is None else t
+    nA, nAcs, nB, nBcs = norms_rows(A), norms_rows(Acs), norms_cols(B), norms_cols(Bcs)
+    eps_col = np.zeros((M // bs, N))
+    eps_row = np.zeros((M, N // bs))
+    eps_corner = np.zeros((M // bs, N // bs))
+    lib().oracle_sea_bounds(M, N, K, bs, t, _p(nA), _p(nAcs), _p(nB), _p(nBcs), _p(eps_col),
+                            _p(eps_row), _p(eps_corner))
+    return dict(eps_col=eps_col, eps_row=eps_row, eps_corner=eps_corner, nA=nA, nAcs=nAcs,
+                nB=nB, nBcs=nBcs)
+
+
 # ---------------------------------------------------------------- whole path
 def encode(A, B, bs, p):
     Acs = encode_cols(A, bs)
@@ -235,7 +307,8 @@ def encode(A, B, bs, p):
 def apply_faults(A, B, enc, Cm, Ccol, Crow, faults, fma_model=1):
     """O9: recompute each faulted C_fc element with its fault.  A fault is a dict with keys
     row, col (C_fc coordinates: row >= M -> Ccol row row-M; col >= N -> Crow col col-N),
-    site (0 xor final, 1 xor after k_step, 2 add), k_step, xor_mask, add."""
+    site (0 xor final, 1 xor after k_step, 2 add final, 3 add after k_step, 4 xor of the
+    separately rounded product at k_step -- Alg 3 errorVecMul), k_step, xor_mask, add."""
     M, K = A.shape
     N = B.shape[1]
     for f in faults:
@@ -270,3 +343,26 @@ def protected_matmul(A, B, *, bs, p=2, omega=3.0, t=None, fma_model=1, faults=()
         correct(Cm, Ccol, Crow, K, bs, p, enc["topA"], enc["topB"], res, omega=omega, t=t,
                 fma_model=fma_model)
     return dict(enc=enc, C=Cm, Ccol=Ccol, Crow=Crow, check=res)
+
+
+def abft_matmul_ext(A, B, *, bs, mode="sea", eps_fixed=0.0, t=None, fma_model=1, faults=(),
+                    do_correct=True, nthreads=None):
+    """Comparator paths (NEXT-3): plain checksums (no top-p) + GEMM + check/correct against
+    the SEA-ABFT bound (mode "sea") or one fixed eps (mode "fixed")."""
+    enc = dict(Acs=encode_cols(A, bs), Bcs=encode_rows(B, bs))
+    Cm = gemm(A, B, fma_model, nthreads)
+    Ccol = gemm(enc["Acs"], B, fma_model, nthreads)
+    Crow = gemm(A, enc["Bcs"], fma_model, nthreads)
+    if faults:
+        apply_faults(A, B, enc, Cm, Ccol, Crow, faults, fma_model)
+    if mode == "sea":
+        sea = sea_bounds(A, B, enc["Acs"], enc["Bcs"], bs, t=t)
+        ec, er = sea["eps_col"], sea["eps_row"]
+    elif mode == "fixed":
+        sea, ec, er = None, None, None
+    else:
+        raise ValueError(mode)
+    res = check_ext(Cm, Ccol, Crow, bs, eps_col=ec, eps_row=er, eps_fixed=eps_fixed)
+    if do_correct:
+        correct_ext(Cm, Ccol, Crow, bs, res, eps_row=er, eps_fixed=eps_fixed)
+    return dict(enc=enc, C=Cm, Ccol=Ccol, Crow=Crow, check=res, sea=sea)
