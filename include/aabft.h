@@ -142,11 +142,15 @@ typedef struct {
  * (row, col) are C_fc coordinates: row in [M, M + M/bs) hits Ccol row row-M;
  * col in [N, N + N/bs) hits Crow column col-N.
  *  site 0: XOR xor_mask into the stored result ("errorVecAdd2")
- *  site 1: XOR xor_mask into the accumulator after the k-tile that contains k_step
- *          ("errorVecAdd1" at k-tile granularity; products inside the DMMA unit
- *          are not addressable)
+ *  site 1: XOR xor_mask into the accumulator ("errorVecAdd1").  FP32 (FFMA):
+ *          right after step k_step, instruction-exact.  FP64 (DMMA): after the k-tile
+ *          (16 steps) that contains k_step -- products inside the DMMA unit are not
+ *          addressable (R23)
  *  site 2: add `add` to the stored result (magnitude sweep)
- *  site 3: add `add` to the accumulator after the k-tile that contains k_step
+ *  site 3: add `add` to the accumulator, at the same point as site 1
+ *  site 4: FP32 only ("errorVecMul"): at step k_step the product is rounded on
+ *          its own, XOR-ed with xor_mask and added (c = c + (fl(a*b) ^ mask)); the FP64
+ *          kernel ignores it
  * Capacity: the FP64 kernel applies at most 64 faults per 64 x 64 tile of C / Ccol / Crow, the
  * FP32 kernel at most 256 per 128 x 128 tile (i.e. one per 8 x 8 block); extra faults in the
  * same tile are ignored. */
@@ -167,7 +171,10 @@ size_t aabft_workspace_bytes(const aabft_config *cfg);
 /* Step 1 (Alg 1).  A (lda >= K) or B (ldb >= N) may be NULL to encode only the
  * other; the corresponding outputs are then untouched.  Checksums are summed sequentially
  * in ascending order in the working precision, so Acs/Bcs, top-p values and hence every
- * bound are bit-identical to the definition (reading R11). */
+ * bound are bit-identical to the definition (reading R11).
+ * topA_val and topA_idx (likewise topB_*) both NULL: checksums only, no top-p selection --
+ * the encoding of the fixed-eps and SEA-ABFT comparators (Table I); setting only
+ * one of the pair is AABFT_EINVAL. */
 aabft_status aabft_encode(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
                           int64_t ldb, const aabft_encoded *out, void *ws, size_t ws_bytes,
                           void *stream);
@@ -212,6 +219,39 @@ aabft_status aabft_check(const aabft_config *cfg, const aabft_encoded *enc,
 aabft_status aabft_correct(const aabft_config *cfg, const aabft_encoded *enc,
                            const aabft_product *prod, aabft_block_report *reports,
                            aabft_counts *counts, void *stream);
+
+/* ---- NEXT-3 comparators (reporting only; the A-ABFT path above does not use them) ----------
+ *
+ * SEA-ABFT bound (§III, ref [28]) for every carried checksum:
+ *   eps = ((n + 2m - 2) ||b||_2 sum_{i=1..m} ||a_i||_2 + n ||a_{m+1}||_2 ||b||_2) 2^-t
+ * with n = K, m = bs: column checksum (I, j) -- a_i the bs rows of block-row I of A, a_{m+1}
+ * = Acs[I], b = column j of B; row checksum (i, J) -- the transposed statement (a_i the bs
+ * columns of block-column J of B, a_{m+1} = Bcs[:, J], b = row i of A); corner (I, J) --
+ * a_{m+1} = Acs[I], b = Bcs[:, J] (reading R25; only for the Table II/III average).  Norms are
+ * sequential ascending sums of squares in double (bit-identical to the definition).  Needs
+ * A, B and the checksums of aabft_encode (top-p not needed).  eps_col: (M/bs) x N, eps_row:
+ * M x (N/bs), eps_corner: (M/bs) x (N/bs), dense doubles, each may be NULL (not all).
+ * ws: the aabft_workspace_bytes(cfg) workspace (holds the norms). */
+aabft_status aabft_sea_bound(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
+                             int64_t ldb, const aabft_encoded *enc, double *eps_col,
+                             double *eps_row, double *eps_corner, void *ws, size_t ws_bytes,
+                             void *stream);
+
+/* Check (Eq 4-6) and correction against an EXTERNAL eps instead of the A-ABFT bound (reading
+ * R26): eps_col ((M/bs) x N) / eps_row (M x (N/bs)) dense device arrays -- e.g. from
+ * aabft_sea_bound -- or, where an array is NULL, eps_fixed for every such check ("ABFT with
+ * manually set error bounds", Table I).  An external eps carries no sigma: classes
+ * are ROUNDING (|d| <= eps) and CRITICAL only.  Verdicts, reports, counts, fused reference
+ * sums (prod->Rcol/Rrow + ws) and the correction rule are those of aabft_check /
+ * aabft_correct; eps_fixed must be >= 0.  The fused reference sums may be checked any number
+ * of times (A-ABFT and comparators over the same product). */
+aabft_status aabft_check_ext(const aabft_config *cfg, const aabft_product *prod,
+                             const double *eps_col, const double *eps_row, double eps_fixed,
+                             aabft_block_report *reports, aabft_counts *counts, void *ws,
+                             size_t ws_bytes, void *stream);
+aabft_status aabft_correct_ext(const aabft_config *cfg, const aabft_product *prod,
+                               const double *eps_row, double eps_fixed,
+                               aabft_block_report *reports, aabft_counts *counts, void *stream);
 
 /* Bound-quality study (NEXT-1; §VI-B, Tables II/III): the signed rounding error of
  * every carried checksum, err = carried - exact, where the exact inner product of the checksum

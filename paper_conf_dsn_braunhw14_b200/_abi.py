@@ -23,7 +23,8 @@ EXPORTED = ("aabft_workspace_bytes", "aabft_encode", "aabft_bound", "aabft_bound
             "aabft_gemm",
             "aabft_gemm_plain", "aabft_check", "aabft_correct", "aabft_host_arena_bytes",
             "aabft_protected_gemm_host", "aabft_status_str", "aabft_last_error",
-            "aabft_version", "aabft_launch_count", "aabft_checksum_errors")
+            "aabft_version", "aabft_launch_count", "aabft_checksum_errors", "aabft_sea_bound",
+            "aabft_check_ext", "aabft_correct_ext")
 
 
 class Config(C.Structure):
@@ -103,6 +104,11 @@ def lib():
         L.aabft_check.argtypes = [pc, C.POINTER(Encoded), C.POINTER(Product), vp, vp, vp, sz, vp]
         L.aabft_correct.argtypes = [pc, C.POINTER(Encoded), C.POINTER(Product), vp, vp, vp]
         L.aabft_protected_gemm_host.argtypes = [pc, vp, vp, vp, vp, vp, sz, vp]
+        L.aabft_sea_bound.argtypes = [pc, vp, i64, vp, i64, C.POINTER(Encoded), vp, vp, vp, vp,
+                                      sz, vp]
+        L.aabft_check_ext.argtypes = [pc, C.POINTER(Product), vp, vp, C.c_double, vp, vp, vp, sz,
+                                      vp]
+        L.aabft_correct_ext.argtypes = [pc, C.POINTER(Product), vp, C.c_double, vp, vp, vp]
         L.aabft_status_str.argtypes = [C.c_int]
         L.aabft_status_str.restype = C.c_char_p
         L.aabft_last_error.restype = C.c_char_p
@@ -110,7 +116,8 @@ def lib():
         L.aabft_launch_count.restype = i64
         for name in ("aabft_encode", "aabft_bound", "aabft_bound_elements", "aabft_checksum_errors",
                      "aabft_gemm", "aabft_gemm_plain",
-                     "aabft_check", "aabft_correct", "aabft_protected_gemm_host"):
+                     "aabft_check", "aabft_correct", "aabft_protected_gemm_host",
+                     "aabft_sea_bound", "aabft_check_ext", "aabft_correct_ext"):
             getattr(L, name).restype = C.c_int
         _lib = L
     return _lib

@@ -131,6 +131,10 @@ class ProtectedGemm:
         self.enc = Encoded(self._Acs.data_ptr(), self.ld_acs, self._Bcs.data_ptr(), self.ld_bcs,
                            self.topA_val.data_ptr(), self.topA_idx.data_ptr(),
                            self.topB_val.data_ptr(), self.topB_idx.data_ptr())
+        # checksums-only view (no top-p tables): the comparators' encoding (NEXT-3)
+        self.enc_cs = Encoded(self._Acs.data_ptr(), self.ld_acs, self._Bcs.data_ptr(),
+                              self.ld_bcs, None, None, None, None)
+        self._sea = None
         # fused check (FP64, bs <= 64): the GEMM epilogue writes the reference sums
         self.fused = bool(fused and dtype == torch.float64 and bs <= 64)
         self.Rcol = torch.empty(nI, N, dtype=torch.float64, device=dev) if self.fused else None
@@ -166,11 +170,13 @@ class ProtectedGemm:
             raise ValueError(f"{name} must be row-major (stride(1) == 1)")
 
     # --- the four steps (each one C-ABI call)
-    def encode(self, A, B, stream=None):
+    def encode(self, A, B, stream=None, topp: bool = True):
+        """Step 1; topp=False encodes the checksums only (fixed-eps / SEA comparators)."""
         L = lib()
         s = _stream_ptr(stream)
         ok(L.aabft_encode(C.byref(self.cfg), _ptr(A), A.stride(0) if A is not None else 0,
-                          _ptr(B), B.stride(0) if B is not None else 0, C.byref(self.enc),
+                          _ptr(B), B.stride(0) if B is not None else 0,
+                          C.byref(self.enc if topp else self.enc_cs),
                           self.ws.data_ptr(), self.ws_bytes, s), "aabft_encode")
 
     def gemm(self, A, B, faults: torch.Tensor | None = None, nfaults: int = 0, stream=None):
@@ -222,6 +228,60 @@ class ProtectedGemm:
                                        err_col.data_ptr(), err_row.data_ptr(), _stream_ptr(stream)),
            "aabft_checksum_errors")
         return err_col, err_row
+
+    # --- NEXT-3 comparators (reporting only)
+    def sea_bound(self, A, B, *, corner: bool = False, stream=None) -> dict:
+        """SEA-ABFT eps of every carried checksum (§III); needs encode() first."""
+        nI, nJ = self.M // self.bs, self.N // self.bs
+        if self._sea is None:
+            self._sea = dict(
+                eps_col=torch.empty(nI, self.N, dtype=torch.float64, device=self.device),
+                eps_row=torch.empty(self.M, nJ, dtype=torch.float64, device=self.device),
+                eps_corner=torch.empty(nI, nJ, dtype=torch.float64, device=self.device))
+        d = self._sea
+        ok(lib().aabft_sea_bound(C.byref(self.cfg), A.data_ptr(), A.stride(0), B.data_ptr(),
+                                 B.stride(0), C.byref(self.enc_cs), d["eps_col"].data_ptr(),
+                                 d["eps_row"].data_ptr(),
+                                 d["eps_corner"].data_ptr() if corner else None,
+                                 self.ws.data_ptr(), self.ws_bytes, _stream_ptr(stream)),
+           "aabft_sea_bound")
+        return d
+
+    def check_ext(self, *, eps_col=None, eps_row=None, eps_fixed: float = 0.0, stream=None):
+        ok(lib().aabft_check_ext(C.byref(self.cfg), C.byref(self.prod), _ptr(eps_col),
+                                 _ptr(eps_row), float(eps_fixed), self.reports.data_ptr(),
+                                 self.counts.data_ptr(), self.ws.data_ptr(), self.ws_bytes,
+                                 _stream_ptr(stream)), "aabft_check_ext")
+
+    def correct_ext(self, *, eps_row=None, eps_fixed: float = 0.0, stream=None):
+        ok(lib().aabft_correct_ext(C.byref(self.cfg), C.byref(self.prod), _ptr(eps_row),
+                                   float(eps_fixed), self.reports.data_ptr(),
+                                   self.counts.data_ptr(), _stream_ptr(stream)),
+           "aabft_correct_ext")
+
+    def run_ext(self, A, B, *, mode: str = "sea", eps_fixed: float = 0.0, faults=None,
+                correct: bool = True, stream=None) -> Result:
+        """Comparator paths of Table I: checksums-only encode -> GEMM -> check /
+        correct against the SEA-ABFT bound (mode "sea") or one fixed eps (mode "fixed")."""
+        if mode not in ("sea", "fixed"):
+            raise ValueError(mode)
+        self._check_operand(A, self.M, self.K, "A")
+        self._check_operand(B, self.K, self.N, "B")
+        fbuf = faults if isinstance(faults, torch.Tensor) else make_faults(faults, self.device)
+        nf = 0 if fbuf is None else fbuf.numel() // 48
+        self.encode(A, B, stream, topp=False)
+        ok(lib().aabft_gemm(C.byref(self.cfg), A.data_ptr(), A.stride(0), B.data_ptr(),
+                            B.stride(0), C.byref(self.enc_cs), C.byref(self.prod), _ptr(fbuf),
+                            nf, self.ws.data_ptr(), self.ws_bytes, _stream_ptr(stream)),
+           "aabft_gemm")
+        ec = er = None
+        if mode == "sea":
+            d = self.sea_bound(A, B, stream=stream)
+            ec, er = d["eps_col"], d["eps_row"]
+        self.check_ext(eps_col=ec, eps_row=er, eps_fixed=eps_fixed, stream=stream)
+        if correct:
+            self.correct_ext(eps_row=er, eps_fixed=eps_fixed, stream=stream)
+        return self.result()
 
     def run(self, A, B, *, faults=None, correct: bool = True, stream=None) -> Result:
         """encode -> gemm -> check -> correct, all enqueued on one stream."""

@@ -13,7 +13,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 OUT = os.environ.get("AABFT_BUILD_OUT", os.path.join(HERE, "libaabft.so"))
 OBJ = os.environ.get("AABFT_BUILD_OBJ", os.path.join(HERE, "build"))
-SOURCES = ["api.cu", "encode.cu", "check.cu", "gemm_f64.cu", "gemm_f32.cu", "study.cu"]
+SOURCES = ["api.cu", "encode.cu", "check.cu", "gemm_f64.cu", "gemm_f32.cu", "study.cu", "sea.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC,-ffp-contract=off", "-Xptxas", "-v", "-I", os.path.join(HERE, "..", "include"),

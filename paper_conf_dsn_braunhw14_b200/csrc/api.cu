@@ -105,8 +105,12 @@ static aabft_status device_ok() {
 static size_t gemm_ws_bytes(const aabft_config *c) {
   return c->dtype == AABFT_F64 ? gemm_f64_ws_bytes(c) : 0;
 }
+// [encode partial top-p lists | SEA norms][FP64 GEMM split-K partials + flags]
+static size_t front_ws_bytes(const aabft_config *c) {
+  return r256(std::max(encode_ws_bytes(c), sea_ws_bytes(c)));
+}
 static void *gemm_ws(const aabft_config *c, void *ws) {
-  return static_cast<char *>(ws) + r256(encode_ws_bytes(c));
+  return static_cast<char *>(ws) + front_ws_bytes(c);
 }
 
 static bool pitch_ok(const aabft_config *c, const void *p, int64_t ld) {
@@ -129,8 +133,7 @@ extern "C" {
 
 size_t aabft_workspace_bytes(const aabft_config *cfg) {
   if (validate(cfg) != AABFT_OK) return 0;
-  // [encode partial top-p lists][FP64 GEMM split-K partials + flags]
-  return r256(encode_ws_bytes(cfg)) + r256(gemm_ws_bytes(cfg)) + 256;
+  return front_ws_bytes(cfg) + r256(gemm_ws_bytes(cfg)) + 256;
 }
 
 aabft_status aabft_encode(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
@@ -141,12 +144,13 @@ aabft_status aabft_encode(const aabft_config *cfg, const void *A, int64_t lda, c
   if (s != AABFT_OK) return s;
   if (!out) { set_error("out is NULL"); return AABFT_EINVAL; }
   if (!A && !B) { set_error("A and B are both NULL"); return AABFT_EINVAL; }
-  if (A && (lda < cfg->K || !out->Acs || out->ld_acs < cfg->K || !out->topA_val || !out->topA_idx)) {
-    set_error("encode A: need lda >= K, Acs (ld_acs >= K), topA_val, topA_idx");
+  // top-p tables: both pointers or neither (neither = checksums only, NEXT-3 comparators)
+  if (A && (lda < cfg->K || !out->Acs || out->ld_acs < cfg->K || (!out->topA_val != !out->topA_idx))) {
+    set_error("encode A: need lda >= K, Acs (ld_acs >= K), topA_val and topA_idx both set or both NULL");
     return AABFT_EINVAL;
   }
-  if (B && (ldb < cfg->N || !out->Bcs || out->ld_bcs < cfg->N / cfg->bs || !out->topB_val || !out->topB_idx)) {
-    set_error("encode B: need ldb >= N, Bcs (ld_bcs >= N/bs), topB_val, topB_idx");
+  if (B && (ldb < cfg->N || !out->Bcs || out->ld_bcs < cfg->N / cfg->bs || (!out->topB_val != !out->topB_idx))) {
+    set_error("encode B: need ldb >= N, Bcs (ld_bcs >= N/bs), topB_val and topB_idx both set or both NULL");
     return AABFT_EINVAL;
   }
   if ((A && !pitch_ok(cfg, A, lda)) || (B && !pitch_ok(cfg, B, ldb))) {
@@ -300,6 +304,71 @@ aabft_status aabft_correct(const aabft_config *cfg, const aabft_encoded *enc,
   aabft_status s = check_common(cfg, enc, prod, reports, counts);
   if (s != AABFT_OK) return s;
   return launch_correct(cfg, enc, prod, reports, counts, (cudaStream_t)stream);
+  AABFT_GUARD_END
+}
+
+// ------------------------------------------------------------------ NEXT-3 comparators
+aabft_status aabft_sea_bound(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
+                             int64_t ldb, const aabft_encoded *enc, double *eps_col,
+                             double *eps_row, double *eps_corner, void *ws, size_t ws_bytes,
+                             void *stream) {
+  AABFT_GUARD_BEGIN
+  aabft_status s = validate(cfg);
+  if (s != AABFT_OK) return s;
+  if (!A || !B || !enc || !enc->Acs || !enc->Bcs || lda < cfg->K || ldb < cfg->N ||
+      enc->ld_acs < cfg->K || enc->ld_bcs < cfg->N / cfg->bs) {
+    set_error("sea_bound: A (lda >= K), B (ldb >= N), Acs, Bcs required");
+    return AABFT_EINVAL;
+  }
+  if (!eps_col && !eps_row && !eps_corner) { set_error("sea_bound: no output"); return AABFT_EINVAL; }
+  if (!pitch_ok(cfg, A, lda) || !pitch_ok(cfg, enc->Acs, enc->ld_acs)) {
+    set_error("sea_bound: A / Acs must be 16-byte aligned with 16-byte-multiple row pitches");
+    return AABFT_EINVAL;
+  }
+  if (!ws || ws_bytes < aabft_workspace_bytes(cfg)) {
+    set_error("workspace too small: need %zu bytes", aabft_workspace_bytes(cfg));
+    return AABFT_EWORKSPACE;
+  }
+  if ((s = device_ok()) != AABFT_OK) return s;
+  return launch_sea_bound(cfg, A, lda, B, ldb, enc, eps_col, eps_row, eps_corner, ws,
+                          (cudaStream_t)stream);
+  AABFT_GUARD_END
+}
+
+static aabft_status ext_common(const aabft_config *cfg, const aabft_product *prod,
+                               double eps_fixed, aabft_block_report *rep, aabft_counts *cnt) {
+  aabft_status s = validate(cfg);
+  if (s != AABFT_OK) return s;
+  if (!prod || !prod->C || !prod->Ccol || !prod->Crow || !rep || !cnt) { set_error("check_ext: C, Ccol, Crow, reports, counts required"); return AABFT_EINVAL; }
+  if (prod->ldc < cfg->N || prod->ld_ccol < cfg->N || prod->ld_crow < cfg->N / cfg->bs) { set_error("check_ext: leading dimensions too small"); return AABFT_EINVAL; }
+  if (!(eps_fixed >= 0.0)) { set_error("check_ext: eps_fixed must be >= 0"); return AABFT_EINVAL; }
+  return device_ok();
+}
+
+aabft_status aabft_check_ext(const aabft_config *cfg, const aabft_product *prod,
+                             const double *eps_col, const double *eps_row, double eps_fixed,
+                             aabft_block_report *reports, aabft_counts *counts, void *ws,
+                             size_t ws_bytes, void *stream) {
+  AABFT_GUARD_BEGIN
+  aabft_status s = ext_common(cfg, prod, eps_fixed, reports, counts);
+  if (s != AABFT_OK) return s;
+  const bool fused = prod->Rcol && prod->Rrow && cfg->dtype == AABFT_F64 && cfg->bs <= 64;
+  if (fused && (!ws || ws_bytes < aabft_workspace_bytes(cfg))) {
+    set_error("check_ext (fused): the aabft_gemm workspace is required");
+    return AABFT_EWORKSPACE;
+  }
+  return launch_check_ext(cfg, prod, eps_col, eps_row, eps_fixed, reports, counts,
+                          fused ? gemm_ws(cfg, ws) : nullptr, (cudaStream_t)stream);
+  AABFT_GUARD_END
+}
+
+aabft_status aabft_correct_ext(const aabft_config *cfg, const aabft_product *prod,
+                               const double *eps_row, double eps_fixed,
+                               aabft_block_report *reports, aabft_counts *counts, void *stream) {
+  AABFT_GUARD_BEGIN
+  aabft_status s = ext_common(cfg, prod, eps_fixed, reports, counts);
+  if (s != AABFT_OK) return s;
+  return launch_correct_ext(cfg, prod, eps_row, eps_fixed, reports, counts, (cudaStream_t)stream);
   AABFT_GUARD_END
 }
 

@@ -154,7 +154,39 @@ struct CheckArgs {
   const double *Rcol2;  // further partial reference sums from the epilogue, added in order
   const double *Rrow2;  // (Rrow2 holds row_parts - 1 planes of M x N/bs)
   int col_parts, row_parts;
+  // external eps (NEXT-3 comparators, reading R26): per-checksum arrays or one fixed value
+  const double *eps_col;  // (M/bs) x N dense, or NULL
+  const double *eps_row;  // M x (N/bs) dense, or NULL
+  double eps_fixed;
 };
+
+// Bound of column check (I, j) / row check (i, J): the A-ABFT bound from the top-p tables, or
+// (EXT) the caller's eps with sigma = eps (an external bound carries no sigma: classes
+// ROUNDING / CRITICAL only, as the oracle's check_ext)
+template <bool EXT, int P>
+__device__ __forceinline__ Bound col_bound(const CheckArgs &a, const BoundParams &bp, int64_t I,
+                                           int64_t j) {
+  if (EXT) {
+    Bound b;
+    b.eps = a.eps_col ? a.eps_col[I * a.N + j] : a.eps_fixed;
+    b.sig = b.eps;
+    return b;
+  }
+  return bound_of(bp, y_bound<P>(a.tav + (a.M + I) * P, a.tai + (a.M + I) * P, a.tbv + j * P,
+                                 a.tbi + j * P));
+}
+template <bool EXT, int P>
+__device__ __forceinline__ Bound row_bound(const CheckArgs &a, const BoundParams &bp, int64_t i,
+                                           int64_t J) {
+  if (EXT) {
+    Bound b;
+    b.eps = a.eps_row ? a.eps_row[i * (a.N / a.bs) + J] : a.eps_fixed;
+    b.sig = b.eps;
+    return b;
+  }
+  return bound_of(bp, y_bound<P>(a.tav + i * P, a.tai + i * P, a.tbv + (a.N + J) * P,
+                                 a.tbi + (a.N + J) * P));
+}
 
 // block verdict + report + aggregated counter update (shared by both check kernels)
 __device__ __forceinline__ void finish_block(const CheckArgs &a, int64_t blk, int nr, int nc,
@@ -186,7 +218,7 @@ __device__ __forceinline__ void finish_block(const CheckArgs &a, int64_t blk, in
                           (unsigned long long)__double_as_longlong(br));
 }
 
-template <typename T, int P>
+template <typename T, int P, bool EXT>
 __global__ void __launch_bounds__(kCheckThreads) check_kernel(CheckArgs a, BoundParams bp) {
   extern __shared__ double tile[];  // kCheckStrip x (bs + 1)
   __shared__ int s_cls[3], s_nr, s_nc, s_row, s_col;
@@ -219,9 +251,7 @@ __global__ void __launch_bounds__(kCheckThreads) check_kernel(CheckArgs a, Bound
       for (int cc = 0; cc < bs; ++cc) ref = ref + tile[row_worker * stride + cc];  // asc j
       const double carried = (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
       const double d = ref - carried;
-      const double y = y_bound<P>(a.tav + i * P, a.tai + i * P, a.tbv + (a.N + J) * P,
-                                  a.tbi + (a.N + J) * P);
-      const Bound b = bound_of(bp, y);
+      const Bound b = row_bound<EXT, P>(a, bp, i, J);
       const int cl = classify(d, b);
       cls_local[cl] += 1;
       if (cl == 2) { atomicAdd(&s_nr, 1); s_row = (int)i; }
@@ -233,9 +263,7 @@ __global__ void __launch_bounds__(kCheckThreads) check_kernel(CheckArgs a, Bound
     const int64_t j = J * bs + tid;
     const double carried = (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
     const double d = colsum - carried;
-    const double y = y_bound<P>(a.tav + (a.M + I) * P, a.tai + (a.M + I) * P, a.tbv + j * P,
-                                a.tbi + j * P);
-    const Bound b = bound_of(bp, y);
+    const Bound b = col_bound<EXT, P>(a, bp, I, j);
     const int cl = classify(d, b);
     cls_local[cl] += 1;
     if (cl == 2) { atomicAdd(&s_nc, 1); s_col = (int)j; }
@@ -266,7 +294,7 @@ __global__ void __launch_bounds__(kCheckThreads) check_kernel(CheckArgs a, Bound
 // carried checksums: 2*bs checks per block, no pass over C.  One WARP per block (grid-stride),
 // warp-shuffle reductions for the verdict, and the counters aggregated per CTA so the device
 // counters see one atomic per CTA instead of one per block.
-template <typename T, int P>
+template <typename T, int P, bool EXT>
 __global__ void __launch_bounds__(256) check_fused_kernel(CheckArgs a, BoundParams bp, int64_t nb) {
   __shared__ unsigned long long s_n[8];
   __shared__ unsigned long long s_mr;
@@ -288,10 +316,10 @@ __global__ void __launch_bounds__(256) check_fused_kernel(CheckArgs a, BoundPara
     const T *ccol_p = static_cast<const T *>(a.Ccol) + I * a.ld_ccol + J * bs;
     const double *rrow = a.Rrow + (I * bs) * nJ + J;
     const T *crow_p = static_cast<const T *>(a.Crow) + (I * bs) * a.ld_crow + J;
-    const double *tva_c = a.tav + (a.M + I) * P;
-    const int *tia_c = a.tai + (a.M + I) * P;
-    const double *tvb_r = a.tbv + (a.N + J) * P;
-    const int *tib_r = a.tbi + (a.N + J) * P;
+    const double *tva_c = EXT ? nullptr : a.tav + (a.M + I) * P;
+    const int *tia_c = EXT ? nullptr : a.tai + (a.M + I) * P;
+    const double *tvb_r = EXT ? nullptr : a.tbv + (a.N + J) * P;
+    const int *tib_r = EXT ? nullptr : a.tbi + (a.N + J) * P;
     int cls[3] = {0, 0, 0}, nr = 0, nc = 0, crow = -1, ccol = -1;
     double rmax = 0.0;
     for (int e = lane; e < 2 * bs; e += 32) {
@@ -300,12 +328,14 @@ __global__ void __launch_bounds__(256) check_fused_kernel(CheckArgs a, BoundPara
       if (e < bs) {  // column check j
         const int j = J32 * bs + e;
         double ref = rcol[e];
-        if (rcol2) {  // complete the epilogue parts (and leave the full sum in Rcol)
-          ref = ref + rcol2[e];
-          const_cast<double *>(rcol)[e] = ref;
+        if (rcol2) {  // complete the epilogue parts (and leave the full sum in Rcol); the
+          ref = ref + rcol2[e];  // consumed part is zeroed so a second check (another bound)
+          const_cast<double *>(rcol)[e] = ref;  // over the same product sees the same sums
+          const_cast<double *>(rcol2)[e] = 0.0;
         }
         d = ref - (double)ccol_p[e];
-        b = bound_of(bp, y_bound<P>(tva_c, tia_c, a.tbv + (int64_t)j * P, a.tbi + (int64_t)j * P));
+        if (EXT) b = col_bound<true, P>(a, bp, I, j);
+        else b = bound_of(bp, y_bound<P>(tva_c, tia_c, a.tbv + (int64_t)j * P, a.tbi + (int64_t)j * P));
         const int cl = classify(d, b);
         cls[cl] += 1;
         if (cl == 2) { nc += 1; ccol = (int)j; }
@@ -314,11 +344,16 @@ __global__ void __launch_bounds__(256) check_fused_kernel(CheckArgs a, BoundPara
         const int64_t i = I * bs + ii;
         double ref = rrow[(int64_t)ii * nJ];
         if (a.row_parts > 1) {
-          for (int q = 1; q < a.row_parts; ++q) ref = ref + a.Rrow2[(q - 1) * a.M * nJ + i * nJ + J];
+          for (int q = 1; q < a.row_parts; ++q) {
+            double *part = const_cast<double *>(a.Rrow2) + (q - 1) * a.M * nJ + i * nJ + J;
+            ref = ref + *part;
+            *part = 0.0;
+          }
           const_cast<double *>(rrow)[(int64_t)ii * nJ] = ref;
         }
         d = ref - (double)crow_p[(int64_t)ii * a.ld_crow];
-        b = bound_of(bp, y_bound<P>(a.tav + i * P, a.tai + i * P, tvb_r, tib_r));
+        if (EXT) b = row_bound<true, P>(a, bp, i, J);
+        else b = bound_of(bp, y_bound<P>(a.tav + i * P, a.tai + i * P, tvb_r, tib_r));
         const int cl = classify(d, b);
         cls[cl] += 1;
         if (cl == 2) { nr += 1; crow = (int)i; }
@@ -373,7 +408,7 @@ __global__ void __launch_bounds__(256) check_fused_kernel(CheckArgs a, BoundPara
 }
 
 // --------------------------------------------------------------------------- correct
-template <typename T, int P>
+template <typename T, int P, bool EXT>
 __global__ void correct_kernel(CheckArgs a, BoundParams bp, T *C) {
   const int bs = a.bs;
   const int64_t nJ = a.N / bs, nb = (a.M / bs) * nJ;
@@ -391,9 +426,7 @@ __global__ void correct_kernel(CheckArgs a, BoundParams bp, T *C) {
     double ref = 0.0;
     for (int64_t jj = J * bs; jj < J * bs + bs; ++jj) ref = ref + (double)C[i * a.ldc + jj];
     const double d = ref - (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
-    const double y = y_bound<P>(a.tav + i * P, a.tai + i * P, a.tbv + (a.N + J) * P,
-                                a.tbi + (a.N + J) * P);
-    const Bound b = bound_of(bp, y);
+    const Bound b = row_bound<EXT, P>(a, bp, i, J);
     unsigned long long *n = reinterpret_cast<unsigned long long *>(a.cnt->n);
     if (fabs(d) <= b.eps) {
       r->status = AABFT_BLK_CORRECTED;
@@ -412,8 +445,8 @@ CheckArgs make_args(const aabft_config *cfg, const aabft_encoded *enc, const aab
   a.C = prod->C; a.ldc = prod->ldc;
   a.Ccol = prod->Ccol; a.ld_ccol = prod->ld_ccol;
   a.Crow = prod->Crow; a.ld_crow = prod->ld_crow;
-  a.tav = enc->topA_val; a.tai = enc->topA_idx;
-  a.tbv = enc->topB_val; a.tbi = enc->topB_idx;
+  a.tav = enc ? enc->topA_val : nullptr; a.tai = enc ? enc->topA_idx : nullptr;
+  a.tbv = enc ? enc->topB_val : nullptr; a.tbi = enc ? enc->topB_idx : nullptr;
   a.rep = rep; a.cnt = cnt;
   // fused reference sums exist only where aabft_gemm produces them (FP64, bs <= 64)
   const bool fused = prod->Rcol && prod->Rrow && cfg->dtype == AABFT_F64 && cfg->bs <= 64;
@@ -421,6 +454,8 @@ CheckArgs make_args(const aabft_config *cfg, const aabft_encoded *enc, const aab
   a.Rrow = fused && gemm_ws ? prod->Rrow : nullptr;
   a.Rcol2 = a.Rrow2 = nullptr;
   a.col_parts = a.row_parts = 1;
+  a.eps_col = a.eps_row = nullptr;
+  a.eps_fixed = 0.0;
   if (a.Rcol) {
     a.col_parts = gemm_f64_fused_parts(cfg->bs, &a.row_parts);
     double *rc2, *rr2;
@@ -431,19 +466,19 @@ CheckArgs make_args(const aabft_config *cfg, const aabft_encoded *enc, const aab
   return a;
 }
 
-template <typename T, int P>
+template <typename T, int P, bool EXT = false>
 aabft_status run_check(const aabft_config *cfg, const CheckArgs &a, BoundParams bp,
                        cudaStream_t st) {
   const int64_t nb = (cfg->M / cfg->bs) * (cfg->N / cfg->bs);
   const size_t smem = (size_t)kCheckStrip * (cfg->bs + 1) * sizeof(double);
-  auto kern = check_kernel<T, P>;
+  auto kern = check_kernel<T, P, EXT>;
   if (smem > 48 * 1024) {
     cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   }
   if (nb > 0) {
     if (a.Rcol && a.Rrow) {
       const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((nb + 7) / 8, 148 * 8));
-      check_fused_kernel<T, P><<<grid, 256, 0, st>>>(a, bp, nb);
+      check_fused_kernel<T, P, EXT><<<grid, 256, 0, st>>>(a, bp, nb);
     } else {
       kern<<<(unsigned)nb, kCheckThreads, smem, st>>>(a, bp);
     }
@@ -452,13 +487,13 @@ aabft_status run_check(const aabft_config *cfg, const CheckArgs &a, BoundParams 
   return check_launch("aabft_check");
 }
 
-template <typename T, int P>
+template <typename T, int P, bool EXT = false>
 aabft_status run_correct(const aabft_config *cfg, const CheckArgs &a, BoundParams bp,
                          cudaStream_t st) {
   const int64_t nb = (cfg->M / cfg->bs) * (cfg->N / cfg->bs);
   const unsigned grid = (unsigned)std::min<int64_t>((nb + 255) / 256, 4096);
   if (nb > 0) {
-    correct_kernel<T, P><<<grid, 256, 0, st>>>(a, bp, static_cast<T *>(const_cast<void *>(a.C)));
+    correct_kernel<T, P, EXT><<<grid, 256, 0, st>>>(a, bp, static_cast<T *>(const_cast<void *>(a.C)));
     next_launch();
   }
   return check_launch("aabft_correct");
@@ -559,6 +594,34 @@ aabft_status launch_correct(const aabft_config *cfg, const aabft_encoded *enc,
   }
   set_error("p out of range");
   return AABFT_EINVAL;
+}
+
+// check / correct against an external eps (NEXT-3 comparators: SEA-ABFT bound, fixed-eps ABFT;
+// reading R26).  The top-p tables are not used; P = 1 instantiations.
+aabft_status launch_check_ext(const aabft_config *cfg, const aabft_product *prod,
+                              const double *eps_col, const double *eps_row, double eps_fixed,
+                              aabft_block_report *rep, aabft_counts *cnt, void *gemm_ws,
+                              cudaStream_t st) {
+  const BoundParams bp = make_bound_params(cfg);
+  CheckArgs a = make_args(cfg, nullptr, prod, rep, cnt, gemm_ws);
+  a.eps_col = eps_col;
+  a.eps_row = eps_row;
+  a.eps_fixed = eps_fixed;
+  if (cudaMemsetAsync(cnt, 0, sizeof(aabft_counts), st) != cudaSuccess)
+    return check_launch("aabft_check_ext memset");
+  if (cfg->dtype == AABFT_F64) return run_check<double, 1, true>(cfg, a, bp, st);
+  return run_check<float, 1, true>(cfg, a, bp, st);
+}
+
+aabft_status launch_correct_ext(const aabft_config *cfg, const aabft_product *prod,
+                                const double *eps_row, double eps_fixed, aabft_block_report *rep,
+                                aabft_counts *cnt, cudaStream_t st) {
+  const BoundParams bp = make_bound_params(cfg);
+  CheckArgs a = make_args(cfg, nullptr, prod, rep, cnt);
+  a.eps_row = eps_row;
+  a.eps_fixed = eps_fixed;
+  if (cfg->dtype == AABFT_F64) return run_correct<double, 1, true>(cfg, a, bp, st);
+  return run_correct<float, 1, true>(cfg, a, bp, st);
 }
 
 }  // namespace aabft

@@ -69,6 +69,18 @@ aabft_status launch_check(const aabft_config *cfg, const aabft_encoded *enc,
 aabft_status launch_correct(const aabft_config *cfg, const aabft_encoded *enc,
                             const aabft_product *prod, aabft_block_report *rep,
                             aabft_counts *cnt, cudaStream_t st);
+// NEXT-3 comparators (check.cu, sea.cu)
+aabft_status launch_check_ext(const aabft_config *cfg, const aabft_product *prod,
+                              const double *eps_col, const double *eps_row, double eps_fixed,
+                              aabft_block_report *rep, aabft_counts *cnt, void *gemm_ws,
+                              cudaStream_t st);
+aabft_status launch_correct_ext(const aabft_config *cfg, const aabft_product *prod,
+                                const double *eps_row, double eps_fixed, aabft_block_report *rep,
+                                aabft_counts *cnt, cudaStream_t st);
+size_t sea_ws_bytes(const aabft_config *cfg);
+aabft_status launch_sea_bound(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
+                              int64_t ldb, const aabft_encoded *enc, double *eps_col,
+                              double *eps_row, double *eps_corner, void *ws, cudaStream_t st);
 
 // ----------------------------------------------------------------------------- device side
 // Top-p list order: value descending, then index ascending (reading R13).  Because indices

@@ -25,7 +25,7 @@ __device__ __forceinline__ T ldg(const T *p) { return __ldg(p); }
 
 // ---------------------------------------------------------------------------------- A
 // grid (chunks of 128 columns, M/bs block-rows); 128 threads.
-template <typename T, int P>
+template <typename T, int P, bool TOPP>
 __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, int64_t lda,
                                                        int64_t K, int bs, T *__restrict__ Acs,
                                                        int64_t ld_acs, double *__restrict__ pv,
@@ -48,9 +48,10 @@ __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, 
     for (int rr = 0; rr < kStrip; ++rr) {
       if (rr < rows) {
         sum = sum + vals[rr];  // Eq 1, ascending i (Alg 1 line "sum <- sum + Asub[i][tid]")
-        tile[rr][c] = fabs((double)vals[rr]);
+        if (TOPP) tile[rr][c] = fabs((double)vals[rr]);
       }
     }
+    if (!TOPP) continue;  // checksums only (fixed-eps / SEA ABFT comparators, NEXT-3)
     __syncthreads();
     double v[P];
     int ix[P];
@@ -75,7 +76,7 @@ __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, 
   }
   if (kin) Acs[I * ld_acs + k] = sum;
   // partial top-p of the checksum row I over this chunk (Alg 1 localSums / maxReduce)
-  {
+  if (TOPP) {
     __shared__ double s_v[kEncAChunk / 32][P];
     __shared__ int s_i[kEncAChunk / 32][P];
     double v[P];
@@ -104,7 +105,7 @@ __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, 
 
 // ---------------------------------------------------------------------------------- B
 // grid (column chunks of NC, row chunks of kEncBChunk); NC threads (NC = max(128, bs)).
-template <typename T, int P, int NC>
+template <typename T, int P, int NC, bool TOPP>
 __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, int64_t ldb,
                                                       int64_t K, int64_t N, int bs,
                                                       T *__restrict__ Bcs, int64_t ld_bcs,
@@ -135,7 +136,7 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
     for (int rr = 0; rr < SB; ++rr) {
       if (rr < rows) {
         tile[rr][c] = vals[rr];
-        if (jin) tp_insert<P>(v, ix, fabs((double)vals[rr]), (int)(k0 + rr));
+        if (TOPP && jin) tp_insert<P>(v, ix, fabs((double)vals[rr]), (int)(k0 + rr));
       }
     }
     __syncthreads();
@@ -152,8 +153,9 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
         T sm = T(0);
         for (int jj = 0; jj < bs; ++jj) sm = sm + tile[rr][jb * bs + jj];
         Bcs[(k0 + rr) * ld_bcs + J] = sm;
-        tp_insert<P>(lv, li, fabs((double)sm), (int)(k0 + rr));
+        if (TOPP) tp_insert<P>(lv, li, fabs((double)sm), (int)(k0 + rr));
       }
+      if (!TOPP) continue;
 #pragma unroll
       for (int m = 16; m >= 1; m >>= 1) tp_shfl_merge<P>(lv, li, m);
       if (rr == 0) {
@@ -165,6 +167,7 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
     }
     __syncthreads();
   }
+  if (!TOPP) return;
   if (c < nblk && ((int64_t)blockIdx.x * nblk + c) * bs < N) {
     const int64_t J = (int64_t)blockIdx.x * nblk + c;
     double *dv = pv + ((N + J) * nch + kc) * P;
@@ -238,29 +241,37 @@ aabft_status run_encode(const aabft_config *cfg, const T *A, int64_t lda, const 
   double *pvb = reinterpret_cast<double *>(w);
   w += (rb * nchb * P * 8 + 255) / 256 * 256;
   int *pib = reinterpret_cast<int *>(w);
+  // top-p tables NULL: checksums only (the encoding of the fixed-eps and SEA comparators)
+  const bool tpa = A && out->topA_val, tpb = B && out->topB_val;
   if (A) {
     dim3 grid(ncha, (unsigned)(M / bs));
-    encode_a_kernel<T, P><<<grid, 128, 0, st>>>(A, lda, K, bs, static_cast<T *>(out->Acs),
-                                                out->ld_acs, pva, pia, ncha);
+    auto kern = tpa ? encode_a_kernel<T, P, true> : encode_a_kernel<T, P, false>;
+    kern<<<grid, 128, 0, st>>>(A, lda, K, bs, static_cast<T *>(out->Acs), out->ld_acs, pva, pia,
+                               ncha);
     next_launch();
   }
   if (B) {
     const int NC = std::max(128, bs);
     dim3 grid((unsigned)((N + NC - 1) / NC), nchb);
-    if (NC == 128)
-      encode_b_kernel<T, P, 128><<<grid, 128, 0, st>>>(B, ldb, K, N, bs, static_cast<T *>(out->Bcs),
-                                                       out->ld_bcs, pvb, pib, nchb);
-    else
-      encode_b_kernel<T, P, 256><<<grid, 256, 0, st>>>(B, ldb, K, N, bs, static_cast<T *>(out->Bcs),
-                                                       out->ld_bcs, pvb, pib, nchb);
+    if (NC == 128) {
+      auto kern = tpb ? encode_b_kernel<T, P, 128, true> : encode_b_kernel<T, P, 128, false>;
+      kern<<<grid, 128, 0, st>>>(B, ldb, K, N, bs, static_cast<T *>(out->Bcs), out->ld_bcs, pvb,
+                                 pib, nchb);
+    } else {
+      auto kern = tpb ? encode_b_kernel<T, P, 256, true> : encode_b_kernel<T, P, 256, false>;
+      kern<<<grid, 256, 0, st>>>(B, ldb, K, N, bs, static_cast<T *>(out->Bcs), out->ld_bcs, pvb,
+                                 pib, nchb);
+    }
     next_launch();
   }
-  const int64_t nvec = (A ? M + M / bs : 0) + (B ? N + N / bs : 0);
-  topp_reduce_kernel<T, P><<<(unsigned)((nvec + 7) / 8), 256, 0, st>>>(
-      M, N, K, bs, pva, pia, ncha, pvb, pib, nchb, static_cast<const T *>(out->Acs), out->ld_acs,
-      static_cast<const T *>(out->Bcs), out->ld_bcs, out->topA_val, out->topA_idx,
-      out->topB_val, out->topB_idx, A != nullptr, B != nullptr);
-  next_launch();
+  const int64_t nvec = (tpa ? M + M / bs : 0) + (tpb ? N + N / bs : 0);
+  if (nvec > 0) {
+    topp_reduce_kernel<T, P><<<(unsigned)((nvec + 7) / 8), 256, 0, st>>>(
+        M, N, K, bs, pva, pia, ncha, pvb, pib, nchb, static_cast<const T *>(out->Acs),
+        out->ld_acs, static_cast<const T *>(out->Bcs), out->ld_bcs, out->topA_val,
+        out->topA_idx, out->topB_val, out->topB_idx, tpa, tpb);
+    next_launch();
+  }
   return check_launch("aabft_encode");
 }
 

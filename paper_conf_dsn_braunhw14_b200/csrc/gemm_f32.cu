@@ -6,8 +6,12 @@
 // (LDGSTS) shared-memory ring, LDS.128 fragments and sm_100 FFMA2 (packed fp32x2 FMA).  Every
 // element accumulates c = fma(a_k, b_k, c) in ascending k, which is exactly the fused
 // sequential inner product of Eq 15 / §IV-D -- the FP32 product is bit-identical to the
-// definition.  Same three tile types as the FP64 kernel (C, Ccol, Crow) and the same fault
-// hooks (site 1 at k-tile granularity, BK = 16).
+// definition.  Same three tile types as the FP64 kernel (C, Ccol, Crow).  Fault injection
+// (Alg 3) is a separate instantiation (FAULTS = true, launched only with a fault
+// list) and is instruction-exact: a thread owning a fault whose k_step falls in the current
+// k-tile replays that k-tile step by step in scalar code -- site 4 rounds the product on its
+// own and XORs it ("errorVecMul"), sites 1 / 3 hit the accumulator right after step k_step
+// ("errorVecAdd1") -- so a faulty FP32 product equals the oracle's dot_fault bit for bit.
 #include "common.cuh"
 
 namespace aabft {
@@ -59,6 +63,7 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
+template <bool FAULTS>
 __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs args) {
   // 3-stage cp.async ring: A tile [128 rows][16 k] (k contiguous, as in memory), B tile
   // [16 k][128 cols].  A fragments are LDS.128 along k (4 k-steps of one row), B fragments
@@ -104,7 +109,7 @@ __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs ar
   const int tid = threadIdx.x, tx = tid % TX, ty = tid / TX;
 
   int nf = 0;
-  if (args.nfaults > 0) {
+  if (FAULTS && args.nfaults > 0) {
     if (tid == 0) s_nf = 0;
     __syncthreads();
     for (int f = tid; f < args.nfaults; f += THREADS) {
@@ -168,6 +173,48 @@ __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs ar
     if (kt + STAGES - 1 < nk) load_tile((kt + STAGES - 1) % STAGES, kt + STAGES - 1);
     cp_async_commit();
     const int cur = kt % STAGES;
+    if (FAULTS && nf > 0) {
+      // this thread's in-loop faults (sites 1, 3, 4) whose k_step falls inside k-tile kt
+      int myf[4], nmy = 0;
+      for (int f = 0; f < nf; ++f) {
+        const aabft_fault &ft = s_f[f];
+        if ((ft.site == 1 || ft.site == 3 || ft.site == 4) && ft.k_step / BK == kt &&
+            ((ft.row & 63) >> 2) == ty && ((ft.col % HN) >> 2) == tx && nmy < 4)
+          myf[nmy++] = f;
+      }
+      if (nmy > 0) {  // scalar replay of this k-tile, step by step (ascending k, as Alg 3)
+        for (int kk = 0; kk < BK; ++kk) {
+          const int64_t k = (int64_t)kt * BK + kk;
+          if (k >= K) break;
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const int r = i < 4 ? ty * 4 + i : 64 + ty * 4 + (i - 4);
+            const float av = As[cur][r][kk];
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+              const int c = j < 4 ? tx * 4 + j : HN + tx * 4 + (j - 4);
+              const float bv = Bs[cur][kk][c];
+              float acc = ACC(i, j);
+              int site = -1;
+              uint64_t mask = 0;
+              double add = 0.0;
+              for (int q = 0; q < nmy; ++q) {
+                const aabft_fault &ft = s_f[myf[q]];
+                if (ft.row == r && ft.col == c && ft.k_step == k) {
+                  site = ft.site; mask = ft.xor_mask; add = ft.add;
+                }
+              }
+              if (site == 4) acc = __fadd_rn(acc, xor_bits(__fmul_rn(av, bv), mask));
+              else acc = __fmaf_rn(av, bv, acc);
+              if (site == 1) acc = xor_bits(acc, mask);
+              if (site == 3) acc = (float)((double)acc + add);
+              ACC(i, j) = acc;
+            }
+          }
+        }
+        continue;
+      }
+    }
 #pragma unroll
     for (int k4 = 0; k4 < BK / 4; ++k4) {
       float4 a4[8];
@@ -190,29 +237,13 @@ __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs ar
         }
       }
     }
-    if (nf > 0) {
-      for (int f = 0; f < nf; ++f) {
-        const aabft_fault ft = s_f[f];
-        if ((ft.site != 1 && ft.site != 3) || ft.k_step / BK != kt) continue;
-#pragma unroll
-        for (int i = 0; i < 8; ++i)
-#pragma unroll
-          for (int j = 0; j < 8; ++j) {
-            const int r = (i < 4 ? ty * 4 + i : 64 + ty * 4 + i - 4);
-            const int c = (j < 4 ? tx * 4 + j : HN + tx * 4 + j - 4);
-            if (r == ft.row && c == ft.col)
-              ACC(i, j) = ft.site == 1 ? xor_bits(ACC(i, j), ft.xor_mask)
-                                       : (float)((double)ACC(i, j) + ft.add);
-          }
-      }
-    }
   }
   cp_async_wait<0>();
 
-  if (nf > 0) {
+  if (FAULTS && nf > 0) {  // sites 0 / 2: the stored result ("errorVecAdd2")
     for (int f = 0; f < nf; ++f) {
       const aabft_fault ft = s_f[f];
-      if (ft.site == 1 || ft.site == 3) continue;
+      if (ft.site != 0 && ft.site != 2) continue;
 #pragma unroll
       for (int i = 0; i < 8; ++i)
 #pragma unroll
@@ -286,12 +317,14 @@ aabft_status launch_gemm_f32(const aabft_config *cfg, const void *A, int64_t lda
   const int64_t tiles = a.n0 + a.n1 + a.n2;
   static bool attr = false;
   if (!attr) {
-    if (cudaFuncSetAttribute(gemm_f32_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM32) != cudaSuccess)
+    if (cudaFuncSetAttribute(gemm_f32_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM32) != cudaSuccess ||
+        cudaFuncSetAttribute(gemm_f32_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM32) != cudaSuccess)
       return check_launch("gemm_f32 smem attribute");
     attr = true;
   }
   if (tiles > 0) {
-    gemm_f32_kernel<<<(unsigned)tiles, THREADS, SMEM32, st>>>(a);
+    if (a.nfaults > 0) gemm_f32_kernel<true><<<(unsigned)tiles, THREADS, SMEM32, st>>>(a);
+    else gemm_f32_kernel<false><<<(unsigned)tiles, THREADS, SMEM32, st>>>(a);
     next_launch();
   }
   return check_launch("aabft_gemm(f32)");

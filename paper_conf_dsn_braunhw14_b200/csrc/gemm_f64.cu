@@ -382,7 +382,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
     if (nf > 0) {
       for (int f = 0; f < nf; ++f) {
         const aabft_fault ft = s_f[f];
-        if (ft.site == 1 || ft.site == 3) continue;
+        if (ft.site != 0 && ft.site != 2) continue;
 #pragma unroll
         for (int mt = 0; mt < MT; ++mt)
 #pragma unroll

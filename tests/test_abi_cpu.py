@@ -114,6 +114,31 @@ def test_workspace_and_null_checks(L):
     assert L.aabft_version().startswith(b"aabft-b200")
 
 
+def test_comparator_entry_points_validate(L):
+    """NEXT-3 comparators: argument checks run before any device access."""
+    from paper_conf_dsn_braunhw14_b200 import _abi
+    cfg = _cfg()
+    enc = _abi.Encoded(16, 256, 16, 4, None, None, None, None)
+    # only one of the top-p pair: invalid
+    half = _abi.Encoded(16, 256, 16, 4, 16, None, None, None)
+    assert L.aabft_encode(C.byref(cfg), 16, 256, None, 0, C.byref(half), 16, 1 << 20, None) == 1
+    # SEA bound: no output / missing operand / workspace too small
+    assert L.aabft_sea_bound(C.byref(cfg), 16, 256, 16, 256, C.byref(enc), None, None, None, 16,
+                             1 << 20, None) == 1
+    assert L.aabft_sea_bound(C.byref(cfg), None, 256, 16, 256, C.byref(enc), 16, None, None, 16,
+                             1 << 20, None) == 1
+    assert L.aabft_sea_bound(C.byref(cfg), 16, 256, 16, 256, C.byref(enc), 16, None, None, 16,
+                             8, None) == 4
+    # external-eps check: negative / NaN eps_fixed, missing buffers
+    prod = _abi.Product(16, 256, 16, 256, 16, 4, None, None)
+    for bad in (-1.0, float("nan")):
+        assert L.aabft_check_ext(C.byref(cfg), C.byref(prod), None, None, bad, 16, 16, None, 0,
+                                 None) == 1
+    assert L.aabft_check_ext(C.byref(cfg), C.byref(prod), None, None, 1.0, None, 16, None, 0,
+                             None) == 1
+    assert L.aabft_correct_ext(C.byref(cfg), None, None, 1.0, 16, 16, None) == 1
+
+
 def test_product_path_has_no_oracle_import():
     """The product package never imports or loads anything under oracle/ (no CPU fallback)."""
     pkg = os.path.join(ROOT, "paper_conf_dsn_braunhw14_b200")
