@@ -21,7 +21,8 @@ import torch
 from . import _abi
 from ._abi import Config, Encoded, Fault, Product, ok, lib
 
-__all__ = ["ProtectedGemm", "protected_matmul", "gemm_plain", "make_faults", "counts_dict"]
+__all__ = ["ProtectedGemm", "protected_matmul", "gemm_plain", "make_faults", "make_faults_arrays",
+           "counts_dict"]
 
 
 def _dtype_code(dt: torch.dtype) -> int:
@@ -58,6 +59,19 @@ def make_faults(faults, device) -> torch.Tensor | None:
         arr[n]["k_step"] = f.get("k_step", 0)
         arr[n]["xor_mask"] = np.uint64(f.get("xor_mask", 0))
         arr[n]["add"] = f.get("add", 0.0)
+    return torch.from_numpy(arr.view(np.uint8).copy()).to(device)
+
+
+def make_faults_arrays(row, col, site, k_step=0, xor_mask=0, add=0.0, device="cuda"):
+    """Vectorised make_faults: equal-length arrays (or scalars) -> device aabft_fault array."""
+    row = np.asarray(row, dtype=np.int64)
+    arr = np.zeros(row.size, dtype=_abi.FAULT_DTYPE)
+    arr["row"] = row
+    arr["col"] = np.asarray(col, dtype=np.int64)
+    arr["site"] = np.asarray(site, dtype=np.int32)
+    arr["k_step"] = np.asarray(k_step, dtype=np.int64)
+    arr["xor_mask"] = np.asarray(xor_mask, dtype=np.uint64)
+    arr["add"] = np.asarray(add, dtype=np.float64)
     return torch.from_numpy(arr.view(np.uint8).copy()).to(device)
 
 
