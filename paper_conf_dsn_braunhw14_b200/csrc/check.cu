@@ -291,120 +291,141 @@ __global__ void __launch_bounds__(kCheckThreads) check_kernel(CheckArgs a, Bound
 
 // --------------------------------------------------------------------------- fused check
 // The GEMM epilogue already produced the reference sums (Rcol, Rrow); compare them with the
-// carried checksums: 2*bs checks per block, no pass over C.  One WARP per block (grid-stride),
-// warp-shuffle reductions for the verdict, and the counters aggregated per CTA so the device
-// counters see one atomic per CTA instead of one per block.
+// carried checksums: 2*bs checks per block, no pass over C.  Latency-bound work, so it is laid
+// out for memory-level parallelism: one THREAD per check, every load independent and
+// coalesced.  A CTA owns a unit of JB = 256/bs adjacent blocks of one block-row I: thread t
+// holds column check j = J0*bs + t and row check (i = I*bs + t/JB, J = J0 + t%JB); the block
+// verdicts are gathered in shared memory (atomics only for the rare non-rounding checks) and
+// the device counters see one atomic per CTA.
+constexpr int kFusedThreads = 256;
+
 template <typename T, int P, bool EXT>
-__global__ void __launch_bounds__(256) check_fused_kernel(CheckArgs a, BoundParams bp, int64_t nb) {
+__global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a, BoundParams bp,
+                                                                    int64_t nunits, int ngrp) {
+  constexpr int MAXJB = kFusedThreads / 8;  // bs >= 8
+  __shared__ int s_nr[MAXJB], s_nc[MAXJB], s_row[MAXJB], s_col[MAXJB], s_worst[MAXJB];
+  __shared__ unsigned s_rmax[MAXJB];  // float bits (non-negative: integer order = value order)
   __shared__ unsigned long long s_n[8];
-  __shared__ unsigned long long s_mr;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (tid < 8) s_n[tid] = 0ull;
-  if (tid == 8) s_mr = 0ull;
-  __syncthreads();
-  const int bs = a.bs;
+  __shared__ unsigned s_mr;
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int bs = a.bs, JB = kFusedThreads / bs;
   const int64_t nJ = a.N / bs;
-  unsigned long long my_n[8] = {0, 0, 0, 0, 0, 0, 0, 0};  // lane 0 of each warp
-  double my_mr = 0.0;
-  const int nJ32 = (int)nJ;
-  for (int blk = blockIdx.x * 8 + warp; blk < (int)nb; blk += gridDim.x * 8) {
-    const int I32 = blk / nJ32, J32 = blk - (blk / nJ32) * nJ32;
-    const int64_t I = I32, J = J32;
-    // per-block base pointers (32-bit offsets inside the block)
-    const double *rcol = a.Rcol + I * a.N + J * bs;
-    const double *rcol2 = a.col_parts > 1 ? a.Rcol2 + I * a.N + J * bs : nullptr;
-    const T *ccol_p = static_cast<const T *>(a.Ccol) + I * a.ld_ccol + J * bs;
-    const double *rrow = a.Rrow + (I * bs) * nJ + J;
-    const T *crow_p = static_cast<const T *>(a.Crow) + (I * bs) * a.ld_crow + J;
-    const double *tva_c = EXT ? nullptr : a.tav + (a.M + I) * P;
-    const int *tia_c = EXT ? nullptr : a.tai + (a.M + I) * P;
-    const double *tvb_r = EXT ? nullptr : a.tbv + (a.N + J) * P;
-    const int *tib_r = EXT ? nullptr : a.tbi + (a.N + J) * P;
-    int cls[3] = {0, 0, 0}, nr = 0, nc = 0, crow = -1, ccol = -1;
-    double rmax = 0.0;
-    for (int e = lane; e < 2 * bs; e += 32) {
-      double d;
-      Bound b;
-      if (e < bs) {  // column check j
-        const int j = J32 * bs + e;
-        double ref = rcol[e];
-        if (rcol2) {  // complete the epilogue parts (and leave the full sum in Rcol); the
-          ref = ref + rcol2[e];  // consumed part is zeroed so a second check (another bound)
-          const_cast<double *>(rcol)[e] = ref;  // over the same product sees the same sums
-          const_cast<double *>(rcol2)[e] = 0.0;
+  if (tid < 8) s_n[tid] = 0ull;
+  if (tid == 8) s_mr = 0u;
+  unsigned long long my_n[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  int cls_tot[3] = {0, 0, 0};
+  float mr = 0.f;
+  const int cseg = bs < 32 ? bs : 32;  // lanes sharing one block among the column checks
+  for (int64_t u = blockIdx.x; u < nunits; u += gridDim.x) {
+    const int64_t I = u / ngrp, J0 = (u % ngrp) * JB;
+    if (tid < JB) {
+      s_nr[tid] = 0; s_nc[tid] = 0; s_row[tid] = -1; s_col[tid] = -1; s_worst[tid] = 0;
+      s_rmax[tid] = 0u;
+    }
+    __syncthreads();
+    // ---- column check (I, j): Rcol (+ the epilogue's second part) vs carried Ccol[I][j]
+    {
+      const int Jl = tid / bs;
+      const int64_t j = J0 * bs + tid;
+      float r = 0.f;
+      if (j < a.N) {
+        double *rc = const_cast<double *>(a.Rcol) + I * a.N + j;
+        double ref = *rc;
+        if (a.col_parts > 1) {  // complete the parts and leave the full sum in Rcol; the
+          double *rc2 = const_cast<double *>(a.Rcol2) + I * a.N + j;  // consumed part is zeroed
+          ref = ref + *rc2;  // so a second check (another bound) sees the same sums
+          *rc = ref;
+          *rc2 = 0.0;
         }
-        d = ref - (double)ccol_p[e];
-        if (EXT) b = col_bound<true, P>(a, bp, I, j);
-        else b = bound_of(bp, y_bound<P>(tva_c, tia_c, a.tbv + (int64_t)j * P, a.tbi + (int64_t)j * P));
+        const double d = ref - (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
+        const Bound b = col_bound<EXT, P>(a, bp, I, j);
         const int cl = classify(d, b);
-        cls[cl] += 1;
-        if (cl == 2) { nc += 1; ccol = (int)j; }
-      } else {  // row check i
-        const int ii = e - bs;
-        const int64_t i = I * bs + ii;
-        double ref = rrow[(int64_t)ii * nJ];
+        cls_tot[cl] += 1;
+        if (cl) {
+          atomicMax(&s_worst[Jl], cl);
+          if (cl == 2) { atomicAdd(&s_nc[Jl], 1); s_col[Jl] = (int)j; }
+        }
+        r = (float)ratio_fast(d, b.eps);
+      }
+      for (int m = 1; m < cseg; m <<= 1) r = fmaxf(r, __shfl_xor_sync(0xffffffffu, r, m));
+      if ((lane & (cseg - 1)) == 0 && r > 0.f) atomicMax(&s_rmax[Jl], __float_as_uint(r));
+    }
+    // ---- row check (i, J): Rrow (+ parts) vs carried Crow[i][J]
+    {
+      const int ii = tid / JB, Jl = tid - (tid / JB) * JB;
+      const int64_t J = J0 + Jl, i = I * bs + ii;
+      float r = 0.f;
+      if (J < nJ) {
+        double *rr = const_cast<double *>(a.Rrow) + i * nJ + J;
+        double ref = *rr;
         if (a.row_parts > 1) {
           for (int q = 1; q < a.row_parts; ++q) {
             double *part = const_cast<double *>(a.Rrow2) + (q - 1) * a.M * nJ + i * nJ + J;
             ref = ref + *part;
             *part = 0.0;
           }
-          const_cast<double *>(rrow)[(int64_t)ii * nJ] = ref;
+          *rr = ref;
         }
-        d = ref - (double)crow_p[(int64_t)ii * a.ld_crow];
-        if (EXT) b = row_bound<true, P>(a, bp, i, J);
-        else b = bound_of(bp, y_bound<P>(a.tav + i * P, a.tai + i * P, tvb_r, tib_r));
+        const double d = ref - (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
+        const Bound b = row_bound<EXT, P>(a, bp, i, J);
         const int cl = classify(d, b);
-        cls[cl] += 1;
-        if (cl == 2) { nr += 1; crow = (int)i; }
+        cls_tot[cl] += 1;
+        if (cl) {
+          atomicMax(&s_worst[Jl], cl);
+          if (cl == 2) { atomicAdd(&s_nr[Jl], 1); s_row[Jl] = (int)i; }
+        }
+        r = (float)ratio_fast(d, b.eps);
       }
-      rmax = fmax(rmax, ratio_fast(d, b.eps));
+      for (int m = JB; m < 32; m <<= 1) r = fmaxf(r, __shfl_xor_sync(0xffffffffu, r, m));
+      if (lane < JB && r > 0.f) atomicMax(&s_rmax[Jl], __float_as_uint(r));
     }
-#pragma unroll
-    for (int m = 16; m >= 1; m >>= 1) {
-      cls[0] += __shfl_xor_sync(0xffffffffu, cls[0], m);
-      cls[1] += __shfl_xor_sync(0xffffffffu, cls[1], m);
-      cls[2] += __shfl_xor_sync(0xffffffffu, cls[2], m);
-      nr += __shfl_xor_sync(0xffffffffu, nr, m);
-      nc += __shfl_xor_sync(0xffffffffu, nc, m);
-      crow = max(crow, __shfl_xor_sync(0xffffffffu, crow, m));
-      ccol = max(ccol, __shfl_xor_sync(0xffffffffu, ccol, m));
-      rmax = fmax(rmax, __shfl_xor_sync(0xffffffffu, rmax, m));
-    }
-    if (lane == 0) {
+    __syncthreads();
+    // ---- block verdicts (warp 0: JB <= 32 blocks)
+    if (tid < JB && J0 + tid < nJ) {
+      const int nr = s_nr[tid], nc = s_nc[tid];
       uint8_t status;
       if (nr == 0 && nc == 0) status = AABFT_BLK_CLEAN;
       else if (nr == 1 && nc == 1) status = AABFT_BLK_SINGLE;
       else if (nr == 0 || nc == 0) status = AABFT_BLK_CHECKSUM_ONLY;
       else status = AABFT_BLK_UNCORRECTABLE;
-      aabft_block_report r;
-      r.status = status;
-      r.worst_class = (uint8_t)(cls[2] ? 2 : (cls[1] ? 1 : 0));
-      r.n_bad_rows = (uint16_t)min(nr, 65535);
-      r.n_bad_cols = (uint16_t)min(nc, 65535);
-      r.reserved = 0;
-      r.row = status == AABFT_BLK_SINGLE ? crow : -1;
-      r.col = status == AABFT_BLK_SINGLE ? ccol : -1;
-      r.max_ratio = (float)rmax;
-      a.rep[blk] = r;
+      aabft_block_report rep;
+      rep.status = status;
+      rep.worst_class = (uint8_t)s_worst[tid];
+      rep.n_bad_rows = (uint16_t)min(nr, 65535);
+      rep.n_bad_cols = (uint16_t)min(nc, 65535);
+      rep.reserved = 0;
+      rep.row = status == AABFT_BLK_SINGLE ? s_row[tid] : -1;
+      rep.col = status == AABFT_BLK_SINGLE ? s_col[tid] : -1;
+      const float br = __uint_as_float(s_rmax[tid]);
+      rep.max_ratio = br;
+      a.rep[I * nJ + J0 + tid] = rep;
       my_n[0] += 1;
       my_n[1] += status == AABFT_BLK_CLEAN;
       my_n[3] += status == AABFT_BLK_CHECKSUM_ONLY;
       my_n[4] += status == AABFT_BLK_UNCORRECTABLE;
-      my_n[5] += cls[0];
-      my_n[6] += cls[1];
-      my_n[7] += cls[2];
-      my_mr = fmax(my_mr, rmax);
+      mr = fmaxf(mr, br);
     }
+    __syncthreads();  // the per-block slots are re-initialised by the next unit
   }
+  // ---- CTA aggregation: one global atomic per non-zero counter
+  my_n[5] = cls_tot[0]; my_n[6] = cls_tot[1]; my_n[7] = cls_tot[2];
+#pragma unroll
+  for (int c = 0; c < 8; ++c) {
+#pragma unroll
+    for (int m = 16; m >= 1; m >>= 1) my_n[c] += __shfl_xor_sync(0xffffffffu, my_n[c], m);
+  }
+#pragma unroll
+  for (int m = 16; m >= 1; m >>= 1) mr = fmaxf(mr, __shfl_xor_sync(0xffffffffu, mr, m));
   if (lane == 0) {
     for (int c = 0; c < 8; ++c)
       if (my_n[c]) atomicAdd(&s_n[c], my_n[c]);
-    if (my_mr > 0.0) atomicMax(&s_mr, (unsigned long long)__double_as_longlong(my_mr));
+    if (mr > 0.f) atomicMax(&s_mr, __float_as_uint(mr));
   }
   __syncthreads();
   if (tid < 8 && s_n[tid]) atomicAdd(reinterpret_cast<unsigned long long *>(a.cnt->n) + tid, s_n[tid]);
-  if (tid == 8 && s_mr) atomicMax(reinterpret_cast<unsigned long long *>(&a.cnt->max_ratio), s_mr);
+  if (tid == 8 && s_mr)
+    atomicMax(reinterpret_cast<unsigned long long *>(&a.cnt->max_ratio),
+              (unsigned long long)__double_as_longlong((double)__uint_as_float(s_mr)));
 }
 
 // --------------------------------------------------------------------------- correct
@@ -477,8 +498,12 @@ aabft_status run_check(const aabft_config *cfg, const CheckArgs &a, BoundParams 
   }
   if (nb > 0) {
     if (a.Rcol && a.Rrow) {
-      const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((nb + 7) / 8, 148 * 8));
-      check_fused_kernel<T, P, EXT><<<grid, 256, 0, st>>>(a, bp, nb);
+      // units of JB = 256/bs adjacent blocks of one block-row (bs <= 64 => JB >= 4)
+      const int JB = kFusedThreads / cfg->bs;
+      const int64_t ngrp = (cfg->N / cfg->bs + JB - 1) / JB;
+      const int64_t nunits = (cfg->M / cfg->bs) * ngrp;
+      const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(nunits, 148 * 6));
+      check_fused_kernel<T, P, EXT><<<grid, kFusedThreads, 0, st>>>(a, bp, nunits, (int)ngrp);
     } else {
       kern<<<(unsigned)nb, kCheckThreads, smem, st>>>(a, bp);
     }
