@@ -60,7 +60,9 @@ __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, 
 #pragma unroll 4
       for (int cc = q; cc < kEncAChunk; cc += 4) {
         const int64_t kk = (int64_t)chunk * kEncAChunk + cc;
-        if (kk < K) tp_insert<P>(v, ix, tile[r][cc], (int)kk);
+        // ascending columns into this lane's own list: a tie with v[P-1] loses, so the
+        // strict compare is an exact reject test
+        if (kk < K && tile[r][cc] > v[P - 1]) tp_insert<P>(v, ix, tile[r][cc], (int)kk);
       }
     }
     tp_shfl_merge<P>(v, ix, 1);
@@ -136,7 +138,10 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
     for (int rr = 0; rr < SB; ++rr) {
       if (rr < rows) {
         tile[rr][c] = vals[rr];
-        if (TOPP && jin) tp_insert<P>(v, ix, fabs((double)vals[rr]), (int)(k0 + rr));
+        if (TOPP && jin) {  // ascending k, own list: strict compare is an exact reject test
+          const double a = fabs((double)vals[rr]);
+          if (a > v[P - 1]) tp_insert<P>(v, ix, a, (int)(k0 + rr));
+        }
       }
     }
     __syncthreads();
