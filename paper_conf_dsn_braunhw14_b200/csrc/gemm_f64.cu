@@ -51,7 +51,10 @@ constexpr int WARPS_N = 64 / WTN;           // warps across the 64-column tile
 constexpr int NCW = 2 * WARPS_N;            // MMA warps per CTA (2 x WARPS_N)
 constexpr int THREADS = NCW * 32;           // MMA threads (named barrier 1)
 constexpr int CTA_THREADS = THREADS + 32;   // + 1 TMA producer warp
-constexpr int CTAS_PER_SM = NCW == 4 ? 3 : 2;  // 15 / 18 warps per SM (128 / <= 102 registers)
+#ifndef AABFT_F64_CTAS
+#define AABFT_F64_CTAS (NCW == 4 ? 3 : 2)
+#endif
+constexpr int CTAS_PER_SM = AABFT_F64_CTAS;  // 15 / 18 warps per SM (128 / <= 102 registers)
 constexpr int COL_PARTS = 2;                // fused column sums: BS=64 spans the 2 warp rows
 constexpr int ROW_PARTS = 64 / WTN;         // fused row sums: BS=64 spans WARPS_N warp columns
 constexpr int A_BYTES = TILE * BK * 8;      // 8 KiB

@@ -373,6 +373,61 @@ def test_full_size_c2_sampled(P, orc):
         assert norm_err(C[I * bs:(I + 1) * bs, J * bs:(J + 1) * bs], ob["C"], Ab, Bb) <= 1e-13
 
 
+@pytest.mark.parametrize("cfg", [
+    # BASELINE configs[2]: 8192^2 FP32 FFMA, wide exponents, BS 64 (bench --workload c3)
+    dict(name="c3", M=8192, N=8192, K=8192, dtype=np.float32, recipe="wide", tol=None),
+    # BASELINE configs[4]: M=N=8192, K=65536 FP64, BS 64 (bench --workload c5 at one GPU)
+    dict(name="c5", M=8192, N=8192, K=65536, dtype=np.float64, recipe="uniform", tol=1e-13),
+], ids=lambda c: c["name"])
+def test_full_size_sampled(P, orc, cfg):
+    """Full-size parity in the bench launch configuration: clean verdicts everywhere, and the
+    oracle recomputes sampled top-p vectors, rows of C and whole BS x BS blocks one by one.
+    FP32 (FFMA, ascending k) is bit-identical; FP64 within 1e-13 of |A||B|."""
+    M, N, K, dt = cfg["M"], cfg["N"], cfg["K"], cfg["dtype"]
+    bs, p = 64, 2
+    A = gen(cfg["recipe"], M, K, 1, 0, dt)
+    B = gen(cfg["recipe"], K, N, 2, 1, dt)
+    plan = P.ProtectedGemm(M, N, K, dtype=TD[dt], bs=bs, p=p)
+    res = plan.run(to_dev(A), to_dev(B))
+    torch.cuda.synchronize()
+    cnt = res.counts()
+    nb = (M // bs) * (N // bs)
+    assert cnt["blocks"] == nb and cnt["clean"] == nb and cnt["checks_critical"] == 0
+    rng = np.random.default_rng(1)
+    tav, tai = host(plan.topA_val), host(plan.topA_idx)
+    tbv, tbi = host(plan.topB_val), host(plan.topB_idx)
+    Acs, Bcs, C = host(plan.Acs), host(plan.Bcs), host(res.C)
+    for i in rng.integers(0, M, 8):
+        v, ix = orc.topp_vector(A[i], p)
+        assert np.array_equal(tav[i], v) and np.array_equal(tai[i], ix)
+    for j in rng.integers(0, N, 8):
+        v, ix = orc.topp_vector(np.ascontiguousarray(B[:, j]), p)
+        assert np.array_equal(tbv[j], v) and np.array_equal(tbi[j], ix)
+    rows = np.sort(rng.integers(0, M, 4))
+    ref = orc.gemm(A[rows], B)
+    if cfg["tol"] is None:
+        assert np.array_equal(C[rows], ref)
+    else:
+        assert norm_err(C[rows], ref, A[rows], B) <= cfg["tol"]
+    nI, nJ = M // bs, N // bs
+    for (I, J) in [(0, 0), (nI - 1, nJ - 1), (int(rng.integers(nI)), int(rng.integers(nJ)))]:
+        Ab = A[I * bs:(I + 1) * bs]
+        Bb = np.ascontiguousarray(B[:, J * bs:(J + 1) * bs])
+        ob = orc.protected_matmul(Ab, Bb, bs=bs, p=p)
+        assert np.array_equal(Acs[I], ob["enc"]["Acs"][0])
+        assert np.array_equal(Bcs[:, J], ob["enc"]["Bcs"][:, 0])
+        assert np.array_equal(tav[M + I], ob["enc"]["topA"][0][bs])
+        assert np.array_equal(tbv[N + J], ob["enc"]["topB"][0][bs])
+        assert ob["check"].status[0, 0] == res.reports()["status"][I, J] == 0
+        Cb = C[I * bs:(I + 1) * bs, J * bs:(J + 1) * bs]
+        if cfg["tol"] is None:
+            assert np.array_equal(Cb, ob["C"])
+        else:
+            assert norm_err(Cb, ob["C"], Ab, Bb) <= cfg["tol"]
+    del plan, res
+    torch.cuda.empty_cache()
+
+
 def test_distributed_single_rank_nccl(P, orc):
     """The distributed driver (row shard + NCCL counter all-reduce) at world size 1."""
     import os
