@@ -1,9 +1,11 @@
 // gemm_f32.cu -- step 2 of A-ABFT (Eq 3) for FP32 on the FFMA pipe (no TF32: a
 // tensor-core TF32 product would change the rounding model the bound assumes, north_star).
 //
-// B200 design: 128 x 128 x 16 CTA tiles, 256 threads, 8 x 8 register
-// micro-tiles split 2 x 2 (rows ty*4 / 64+ty*4, cols tx*4 / 64+tx*4), a 3-stage cp.async
-// (LDGSTS) shared-memory ring, LDS.128 fragments and sm_100 FFMA2 (packed fp32x2 FMA).  Every
+// B200 design: 128 x 128 x 32 CTA tiles, 256 threads, 8 x 8 register
+// micro-tiles split 2 x 2 (rows ty*4 / 64+ty*4, cols tx*4 / 64+tx*4), a 2-stage cp.async
+// (LDGSTS) shared-memory ring, LDS.128 fragments and sm_100 FFMA2 (packed fp32x2 FMA).
+// (BK 32 x 2 stages measured 54.8 TFLOP/s at 8192^3 against 50.4 for BK 16 x 3, 51.2 for
+// 32 x 3, 52.6 for 16 x 4, 49.8 for 48 x 2: half the CTA barriers per FMA, 2 CTAs/SM.)  Every
 // element accumulates c = fma(a_k, b_k, c) in ascending k, which is exactly the fused
 // sequential inner product of Eq 15 / §IV-D -- the FP32 product is bit-identical to the
 // definition.  Same three tile types as the FP64 kernel (C, Ccol, Crow).  Fault injection
@@ -20,12 +22,21 @@ namespace {
 #ifndef AABFT_F32_BN
 #define AABFT_F32_BN 128
 #endif
-constexpr int BM = 128, BN = AABFT_F32_BN, BK = 16, STAGES = 3;
+#ifndef AABFT_F32_BK
+#define AABFT_F32_BK 32
+#endif
+#ifndef AABFT_F32_STAGES
+#define AABFT_F32_STAGES 2
+#endif
+constexpr int BM = 128, BN = AABFT_F32_BN, BK = AABFT_F32_BK, STAGES = AABFT_F32_STAGES;
 constexpr int TX = BN / 8, THREADS = 16 * TX;   // 16 x TX threads, 8 x 8 outputs each
 constexpr int HN = BN / 2;                      // column offset of the second 4-wide half
 constexpr int MAXF = BM * BN / 64;  // faults per tile kept in smem (one per 8x8 block)
 constexpr int SMEM32 = STAGES * (BM + BN) * BK * 4 + MAXF * (int)sizeof(aabft_fault);
-constexpr int GROUP_M = 8;
+#ifndef AABFT_F32_GROUP_M
+#define AABFT_F32_GROUP_M 8
+#endif
+constexpr int GROUP_M = AABFT_F32_GROUP_M;
 
 struct SgemmArgs {
   const float *A;
@@ -65,8 +76,8 @@ __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_gr
 
 template <bool FAULTS>
 __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs args) {
-  // 3-stage cp.async ring: A tile [128 rows][16 k] (k contiguous, as in memory), B tile
-  // [16 k][128 cols].  A fragments are LDS.128 along k (4 k-steps of one row), B fragments
+  // cp.async ring: A tile [128 rows][BK k] (k contiguous, as in memory), B tile
+  // [BK k][128 cols].  A fragments are LDS.128 along k (4 k-steps of one row), B fragments
   // LDS.128 along n; the 8 x 8 micro-tile runs as 32 FFMA2 per k-step (sm_100 packed fp32x2
   // FMA, A broadcast) -- each lane rounded once, exactly fmaf.
   extern __shared__ __align__(16) uint8_t smem32[];
@@ -139,7 +150,7 @@ __global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs ar
 #pragma unroll
     for (int c = 0; c < BM * BK / 4 / THREADS; ++c) {
       const int e = tid + c * THREADS;
-      const int ar = e >> 2, ak = (e & 3) * 4;   // A: row ar, k ak..ak+3
+      const int ar = e / (BK / 4), ak = (e % (BK / 4)) * 4;  // A: row ar, k ak..ak+3
       const int64_t gr = m0 + ar, gk = k0 + ak;
       const int av = (gr < rows_valid && gk < K) ? (int)((K - gk) * 4 < 16 ? (K - gk) * 4 : 16) : 0;
       cp_async16(&As[stage][ar][ak], av ? (const void *)(Ap + gr * lda + gk) : (const void *)Ap, av);
