@@ -106,6 +106,31 @@ __device__ __forceinline__ void tp_insert(double (&v)[P], int (&ix)[P], double v
     if (r == pos) { v[r] = val; ix[r] = idx; }
 }
 
+// Insertion of an element that loses every tie (its index is larger than all indices in the
+// list: a lane scanning its own elements in ascending index order).  For small P it is
+// branch-free -- g[r] = (a > v[r]) is monotone in r, and slot r takes v[r-1] if g[r-1], else a
+// if g[r], else keeps v[r] -- so a warp whose lanes insert at different elements never
+// diverges; larger P falls back to the early-exit insertion.
+template <int P>
+__device__ __forceinline__ void tp_push(double (&v)[P], int (&ix)[P], double a, int idx) {
+  if (P <= 4) {
+    bool g[P];
+#pragma unroll
+    for (int r = 0; r < P; ++r) g[r] = a > v[r];
+#pragma unroll
+    for (int r = P - 1; r >= 1; --r) {
+      const double vr = g[r - 1] ? v[r - 1] : (g[r] ? a : v[r]);
+      const int ir = g[r - 1] ? ix[r - 1] : (g[r] ? idx : ix[r]);
+      v[r] = vr;
+      ix[r] = ir;
+    }
+    v[0] = g[0] ? a : v[0];
+    ix[0] = g[0] ? idx : ix[0];
+  } else {
+    if (a > v[P - 1]) tp_insert<P>(v, ix, a, idx);
+  }
+}
+
 template <int P>
 __device__ __forceinline__ void tp_init(double (&v)[P], int (&ix)[P]) {
 #pragma unroll

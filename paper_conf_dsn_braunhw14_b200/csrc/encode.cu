@@ -42,13 +42,26 @@ __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, 
     const int rows = min(kStrip, bs - r0);
     const T *src = A + (I * bs + r0) * lda + k;
     T vals[kStrip];
+    if (rows == kStrip) {
+      // full strip: the kStrip loads are issued back to back (memory-level parallelism) --
+      // with the per-row guard below, the checksums-only instantiation compiled to
+      // load -> add -> load chains (latency-bound, 2x slower)
 #pragma unroll
-    for (int rr = 0; rr < kStrip; ++rr) vals[rr] = (rr < rows && kin) ? ldg(src + rr * lda) : T(0);
+      for (int rr = 0; rr < kStrip; ++rr) vals[rr] = kin ? ldg(src + rr * lda) : T(0);
 #pragma unroll
-    for (int rr = 0; rr < kStrip; ++rr) {
-      if (rr < rows) {
+      for (int rr = 0; rr < kStrip; ++rr) {
         sum = sum + vals[rr];  // Eq 1, ascending i (Alg 1 line "sum <- sum + Asub[i][tid]")
         if (TOPP) tile[rr][c] = fabs((double)vals[rr]);
+      }
+    } else {
+#pragma unroll
+      for (int rr = 0; rr < kStrip; ++rr) vals[rr] = (rr < rows && kin) ? ldg(src + rr * lda) : T(0);
+#pragma unroll
+      for (int rr = 0; rr < kStrip; ++rr) {
+        if (rr < rows) {
+          sum = sum + vals[rr];
+          if (TOPP) tile[rr][c] = fabs((double)vals[rr]);
+        }
       }
     }
     if (!TOPP) continue;  // checksums only (fixed-eps / SEA ABFT comparators, NEXT-3)
@@ -60,9 +73,8 @@ __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, 
 #pragma unroll 4
       for (int cc = q; cc < kEncAChunk; cc += 4) {
         const int64_t kk = (int64_t)chunk * kEncAChunk + cc;
-        // ascending columns into this lane's own list: a tie with v[P-1] loses, so the
-        // strict compare is an exact reject test
-        if (kk < K && tile[r][cc] > v[P - 1]) tp_insert<P>(v, ix, tile[r][cc], (int)kk);
+        // ascending columns into this lane's own list: the new element loses every tie
+        if (kk < K) tp_push<P>(v, ix, tile[r][cc], (int)kk);
       }
     }
     tp_shfl_merge<P>(v, ix, 1);
@@ -138,9 +150,9 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
     for (int rr = 0; rr < SB; ++rr) {
       if (rr < rows) {
         tile[rr][c] = vals[rr];
-        if (TOPP && jin) {  // ascending k, own list: strict compare is an exact reject test
+        if (TOPP && jin) {  // ascending k, own list: the new element loses every tie
           const double a = fabs((double)vals[rr]);
-          if (a > v[P - 1]) tp_insert<P>(v, ix, a, (int)(k0 + rr));
+          tp_push<P>(v, ix, a, (int)(k0 + rr));
         }
       }
     }
@@ -158,7 +170,7 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
         T sm = T(0);
         for (int jj = 0; jj < bs; ++jj) sm = sm + tile[rr][jb * bs + jj];
         Bcs[(k0 + rr) * ld_bcs + J] = sm;
-        if (TOPP) tp_insert<P>(lv, li, fabs((double)sm), (int)(k0 + rr));
+        if (TOPP) tp_push<P>(lv, li, fabs((double)sm), (int)(k0 + rr));
       }
       if (!TOPP) continue;
 #pragma unroll
