@@ -38,32 +38,33 @@ __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, 
   const bool kin = k < K;
   const int r = c >> 2, q = c & 3;  // top-p role: row r of the strip, column phase q
   T sum = T(0);
-  for (int r0 = 0; r0 < bs; r0 += kStrip) {
+  // register double buffering: the loads of strip r0 + kStrip are issued right after strip r0
+  // has been summed and staged, so they are in flight during its top-p phase
+  T vals[kStrip];
+  auto load_strip = [&](int r0) {
     const int rows = min(kStrip, bs - r0);
     const T *src = A + (I * bs + r0) * lda + k;
-    T vals[kStrip];
     if (rows == kStrip) {
-      // full strip: the kStrip loads are issued back to back (memory-level parallelism) --
-      // with the per-row guard below, the checksums-only instantiation compiled to
-      // load -> add -> load chains (latency-bound, 2x slower)
+      // full strip: the kStrip loads are issued back to back (memory-level parallelism; a
+      // per-row guard made the checksums-only instantiation compile to load -> add chains)
 #pragma unroll
       for (int rr = 0; rr < kStrip; ++rr) vals[rr] = kin ? ldg(src + rr * lda) : T(0);
-#pragma unroll
-      for (int rr = 0; rr < kStrip; ++rr) {
-        sum = sum + vals[rr];  // Eq 1, ascending i (Alg 1 line "sum <- sum + Asub[i][tid]")
-        if (TOPP) tile[rr][c] = fabs((double)vals[rr]);
-      }
     } else {
 #pragma unroll
       for (int rr = 0; rr < kStrip; ++rr) vals[rr] = (rr < rows && kin) ? ldg(src + rr * lda) : T(0);
+    }
+  };
+  load_strip(0);
+  for (int r0 = 0; r0 < bs; r0 += kStrip) {
+    const int rows = min(kStrip, bs - r0);
 #pragma unroll
-      for (int rr = 0; rr < kStrip; ++rr) {
-        if (rr < rows) {
-          sum = sum + vals[rr];
-          if (TOPP) tile[rr][c] = fabs((double)vals[rr]);
-        }
+    for (int rr = 0; rr < kStrip; ++rr) {
+      if (rr < rows) {
+        sum = sum + vals[rr];  // Eq 1, ascending i (Alg 1 line "sum <- sum + Asub[i][tid]")
+        if (TOPP) tile[rr][c] = fabs((double)vals[rr]);
       }
     }
+    if (r0 + kStrip < bs) load_strip(r0 + kStrip);
     if (!TOPP) continue;  // checksums only (fixed-eps / SEA ABFT comparators, NEXT-3)
     __syncthreads();
     double v[P];
@@ -140,12 +141,22 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
   double v[P];
   int ix[P];
   tp_init<P>(v, ix);
-  for (int64_t k0 = kbeg; k0 < kend; k0 += SB) {
+  // register double buffering as in encode A: strip k0 + SB is loaded during the row sums
+  T vals[SB];
+  auto load_strip = [&](int64_t k0) {
     const int rows = (int)(kend - k0 < SB ? kend - k0 : SB);
     const T *src = B + k0 * ldb + j;
-    T vals[SB];
+    if (rows == SB) {
 #pragma unroll
-    for (int rr = 0; rr < SB; ++rr) vals[rr] = (rr < rows && jin) ? ldg(src + rr * ldb) : T(0);
+      for (int rr = 0; rr < SB; ++rr) vals[rr] = jin ? ldg(src + rr * ldb) : T(0);
+    } else {
+#pragma unroll
+      for (int rr = 0; rr < SB; ++rr) vals[rr] = (rr < rows && jin) ? ldg(src + rr * ldb) : T(0);
+    }
+  };
+  if (kbeg < kend) load_strip(kbeg);
+  for (int64_t k0 = kbeg; k0 < kend; k0 += SB) {
+    const int rows = (int)(kend - k0 < SB ? kend - k0 : SB);
 #pragma unroll
     for (int rr = 0; rr < SB; ++rr) {
       if (rr < rows) {
@@ -156,6 +167,7 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
         }
       }
     }
+    if (k0 + SB < kend) load_strip(k0 + SB);
     __syncthreads();
     // Eq 2 row checksums: lane rr of the warp owning block jb sums row rr sequentially
     // (ascending j), then the warp folds the strip's |Bcs| into the running top-p of
