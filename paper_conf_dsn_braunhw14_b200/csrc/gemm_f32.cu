@@ -75,7 +75,10 @@ template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
 template <bool FAULTS>
-__global__ void __launch_bounds__(THREADS, 2) gemm_f32_kernel(const SgemmArgs args) {
+#ifndef AABFT_F32_MINB
+#define AABFT_F32_MINB (THREADS >= 512 ? 1 : 2)
+#endif
+__global__ void __launch_bounds__(THREADS, AABFT_F32_MINB) gemm_f32_kernel(const SgemmArgs args) {
   // cp.async ring: A tile [128 rows][BK k] (k contiguous, as in memory), B tile
   // [BK k][128 cols].  A fragments are LDS.128 along k (4 k-steps of one row), B fragments
   // LDS.128 along n; the 8 x 8 micro-tile runs as 32 FFMA2 per k-step (sm_100 packed fp32x2
