@@ -20,8 +20,6 @@
 namespace aabft {
 namespace {
 
-constexpr int kCheckThreads = 256;
-constexpr int kCheckStrip = 32;
 
 template <int P>
 __device__ __forceinline__ double y_bound(const double *__restrict__ va, const int *__restrict__ ia,
@@ -218,77 +216,6 @@ __device__ __forceinline__ void finish_block(const CheckArgs &a, int64_t blk, in
                           (unsigned long long)__double_as_longlong(br));
 }
 
-template <typename T, int P, bool EXT>
-__global__ void __launch_bounds__(kCheckThreads) check_kernel(CheckArgs a, BoundParams bp) {
-  extern __shared__ double tile[];  // kCheckStrip x (bs + 1)
-  __shared__ int s_cls[3], s_nr, s_nc, s_row, s_col;
-  __shared__ double s_ratio[kCheckThreads / 32];
-  const int bs = a.bs, tid = threadIdx.x, lane = tid & 31;
-  const int64_t nJ = a.N / bs;
-  const int64_t I = blockIdx.x / nJ, J = blockIdx.x % nJ;
-  const T *C = static_cast<const T *>(a.C);
-  if (tid < 3) s_cls[tid] = 0;
-  if (tid == 0) { s_nr = 0; s_nc = 0; s_row = -1; s_col = -1; }
-  const int stride = bs + 1;
-  const int rs = min(bs, kCheckStrip);
-  double colsum = 0.0;
-  int cls_local[3] = {0, 0, 0};
-  double rmax = 0.0;
-  const int row_worker = tid - (kCheckThreads - kCheckStrip);  // last warp sums rows
-  for (int r0 = 0; r0 < bs; r0 += rs) {
-    // coalesced strip load: rs rows x bs columns
-    for (int e = tid; e < rs * bs; e += kCheckThreads) {
-      const int rr = e / bs, cc = e % bs;
-      tile[rr * stride + cc] = (double)C[(I * bs + r0 + rr) * a.ldc + J * bs + cc];
-    }
-    __syncthreads();
-    if (tid < bs) {
-      for (int rr = 0; rr < rs; ++rr) colsum = colsum + tile[rr * stride + tid];  // Eq 4, asc i
-    }
-    if (row_worker >= 0 && row_worker < rs) {
-      const int64_t i = I * bs + r0 + row_worker;
-      double ref = 0.0;
-      for (int cc = 0; cc < bs; ++cc) ref = ref + tile[row_worker * stride + cc];  // asc j
-      const double carried = (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
-      const double d = ref - carried;
-      const Bound b = row_bound<EXT, P>(a, bp, i, J);
-      const int cl = classify(d, b);
-      cls_local[cl] += 1;
-      if (cl == 2) { atomicAdd(&s_nr, 1); s_row = (int)i; }
-      rmax = fmax(rmax, ratio_of(d, b.eps));
-    }
-    __syncthreads();
-  }
-  if (tid < bs) {
-    const int64_t j = J * bs + tid;
-    const double carried = (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
-    const double d = colsum - carried;
-    const Bound b = col_bound<EXT, P>(a, bp, I, j);
-    const int cl = classify(d, b);
-    cls_local[cl] += 1;
-    if (cl == 2) { atomicAdd(&s_nc, 1); s_col = (int)j; }
-    rmax = fmax(rmax, ratio_of(d, b.eps));
-  }
-  // block reductions
-#pragma unroll
-  for (int c = 0; c < 3; ++c) {
-    int v = cls_local[c];
-#pragma unroll
-    for (int m = 16; m >= 1; m >>= 1) v += __shfl_xor_sync(0xffffffffu, v, m);
-    if (lane == 0 && v) atomicAdd(&s_cls[c], v);
-  }
-#pragma unroll
-  for (int m = 16; m >= 1; m >>= 1) rmax = fmax(rmax, __shfl_xor_sync(0xffffffffu, rmax, m));
-  if (lane == 0) s_ratio[tid >> 5] = rmax;
-  __syncthreads();
-  if (tid == 0) {
-    double br = 0.0;
-    for (int w = 0; w < kCheckThreads / 32; ++w) br = fmax(br, s_ratio[w]);
-    const int cls[3] = {s_cls[0], s_cls[1], s_cls[2]};
-    finish_block(a, blockIdx.x, s_nr, s_nc, s_row, s_col, cls, br);
-  }
-}
-
 // --------------------------------------------------------------------------- fused check
 // The GEMM epilogue already produced the reference sums (Rcol, Rrow); compare them with the
 // carried checksums: 2*bs checks per block, no pass over C.  Latency-bound work, so it is laid
@@ -428,6 +355,142 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
               (unsigned long long)__double_as_longlong((double)__uint_as_float(s_mr)));
 }
 
+// --------------------------------------------------------------------------- streaming check
+// Unfused check (FP32, or bs > 64): re-sums C once, streaming.  A CTA owns block-row I x a
+// chunk of CW = max(128, bs) columns (CW/bs blocks); thread c owns column j0 + c: its Eq 4
+// column reference is a register running sum in ascending row order (double, reading R12).
+// Strips of SR rows go through registers (the next strip's loads are issued before this
+// strip's row-sum phase) into shared memory, where task (row r, block jb) forms the Eq 4 row
+// reference by summing its bs elements in ascending j.  Block verdicts are gathered in shared
+// memory; one global atomic per counter per CTA.
+template <typename T, int P, bool EXT, int CW>
+__global__ void __launch_bounds__(CW) check_stream_kernel(CheckArgs a, BoundParams bp) {
+  constexpr int SR = (CW * sizeof(T) > 1024) ? 16 : 32;  // strip rows (static smem <= 48 KiB)
+  constexpr int MAXB = CW / 8;                           // blocks per chunk (bs >= 8)
+  __shared__ T tile[SR][CW + 1];  // odd pitch: row-sum lanes (one row each) hit distinct banks
+  __shared__ int s_nr[MAXB], s_nc[MAXB], s_row[MAXB], s_col[MAXB], s_worst[MAXB];
+  __shared__ unsigned s_rmax[MAXB];
+  __shared__ unsigned long long s_n[8];
+  __shared__ unsigned s_mr;
+  const int c = threadIdx.x, lane = c & 31;
+  const int bs = a.bs;
+  const int64_t I = blockIdx.y, j0 = (int64_t)blockIdx.x * CW;
+  const int ncols = (int)(a.N - j0 < CW ? a.N - j0 : CW);  // multiple of bs
+  const int nbh = ncols / bs;
+  const int64_t nJ = a.N / bs;
+  if (c < MAXB) {
+    s_nr[c] = 0; s_nc[c] = 0; s_row[c] = -1; s_col[c] = -1; s_worst[c] = 0; s_rmax[c] = 0u;
+  }
+  if (c < 8) s_n[c] = 0ull;
+  if (c == 8) s_mr = 0u;
+  const T *C = static_cast<const T *>(a.C);
+  const bool jin = c < ncols;
+  const T *col = C + (I * bs) * a.ldc + j0 + c;
+  T vals[SR];
+  auto load_strip = [&](int r0) {
+    const int rows = bs - r0 < SR ? bs - r0 : SR;
+    const T *src = col + (int64_t)r0 * a.ldc;
+    if (rows == SR) {
+#pragma unroll
+      for (int rr = 0; rr < SR; ++rr) vals[rr] = jin ? src[(int64_t)rr * a.ldc] : T(0);
+    } else {
+#pragma unroll
+      for (int rr = 0; rr < SR; ++rr) vals[rr] = (jin && rr < rows) ? src[(int64_t)rr * a.ldc] : T(0);
+    }
+  };
+  load_strip(0);
+  __syncthreads();  // slot initialisation
+  double colsum = 0.0;
+  int cls_tot[3] = {0, 0, 0};
+  for (int r0 = 0; r0 < bs; r0 += SR) {
+    const int rows = bs - r0 < SR ? bs - r0 : SR;
+#pragma unroll
+    for (int rr = 0; rr < SR; ++rr) {
+      if (rr < rows) {
+        colsum = colsum + (double)vals[rr];  // Eq 4, ascending i
+        tile[rr][c] = vals[rr];
+      }
+    }
+    if (r0 + SR < bs) load_strip(r0 + SR);
+    __syncthreads();
+    for (int t = c; t < rows * nbh; t += CW) {
+      const int r = t % rows, jb = t / rows;
+      const int64_t i = I * bs + r0 + r, J = j0 / bs + jb;
+      double ref = 0.0;
+      for (int jj = 0; jj < bs; ++jj) ref = ref + (double)tile[r][jb * bs + jj];  // asc j
+      const double d = ref - (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
+      const Bound b = row_bound<EXT, P>(a, bp, i, J);
+      const int cl = classify(d, b);
+      cls_tot[cl] += 1;
+      if (cl) {
+        atomicMax(&s_worst[jb], cl);
+        if (cl == 2) { atomicAdd(&s_nr[jb], 1); s_row[jb] = (int)i; }
+      }
+      const float rt = (float)ratio_fast(d, b.eps);
+      if (rt > 0.f) atomicMax(&s_rmax[jb], __float_as_uint(rt));
+    }
+    __syncthreads();  // tile consumed
+  }
+  if (jin) {
+    const int jb = c / bs;
+    const int64_t j = j0 + c;
+    const double d = colsum - (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
+    const Bound b = col_bound<EXT, P>(a, bp, I, j);
+    const int cl = classify(d, b);
+    cls_tot[cl] += 1;
+    if (cl) {
+      atomicMax(&s_worst[jb], cl);
+      if (cl == 2) { atomicAdd(&s_nc[jb], 1); s_col[jb] = (int)j; }
+    }
+    const float rt = (float)ratio_fast(d, b.eps);
+    if (rt > 0.f) atomicMax(&s_rmax[jb], __float_as_uint(rt));
+  }
+  __syncthreads();
+  unsigned long long my_n[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  float mr = 0.f;
+  if (c < nbh) {  // block verdicts (warp 0: nbh <= 16)
+    const int nr = s_nr[c], nc = s_nc[c];
+    uint8_t status;
+    if (nr == 0 && nc == 0) status = AABFT_BLK_CLEAN;
+    else if (nr == 1 && nc == 1) status = AABFT_BLK_SINGLE;
+    else if (nr == 0 || nc == 0) status = AABFT_BLK_CHECKSUM_ONLY;
+    else status = AABFT_BLK_UNCORRECTABLE;
+    aabft_block_report rep;
+    rep.status = status;
+    rep.worst_class = (uint8_t)s_worst[c];
+    rep.n_bad_rows = (uint16_t)min(nr, 65535);
+    rep.n_bad_cols = (uint16_t)min(nc, 65535);
+    rep.reserved = 0;
+    rep.row = status == AABFT_BLK_SINGLE ? s_row[c] : -1;
+    rep.col = status == AABFT_BLK_SINGLE ? s_col[c] : -1;
+    mr = __uint_as_float(s_rmax[c]);
+    rep.max_ratio = mr;
+    a.rep[I * nJ + j0 / bs + c] = rep;
+    my_n[0] = 1;
+    my_n[1] = status == AABFT_BLK_CLEAN;
+    my_n[3] = status == AABFT_BLK_CHECKSUM_ONLY;
+    my_n[4] = status == AABFT_BLK_UNCORRECTABLE;
+  }
+  my_n[5] = cls_tot[0]; my_n[6] = cls_tot[1]; my_n[7] = cls_tot[2];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+#pragma unroll
+    for (int m = 16; m >= 1; m >>= 1) my_n[k] += __shfl_xor_sync(0xffffffffu, my_n[k], m);
+  }
+#pragma unroll
+  for (int m = 16; m >= 1; m >>= 1) mr = fmaxf(mr, __shfl_xor_sync(0xffffffffu, mr, m));
+  if (lane == 0) {
+    for (int k = 0; k < 8; ++k)
+      if (my_n[k]) atomicAdd(&s_n[k], my_n[k]);
+    if (mr > 0.f) atomicMax(&s_mr, __float_as_uint(mr));
+  }
+  __syncthreads();
+  if (c < 8 && s_n[c]) atomicAdd(reinterpret_cast<unsigned long long *>(a.cnt->n) + c, s_n[c]);
+  if (c == 8 && s_mr)
+    atomicMax(reinterpret_cast<unsigned long long *>(&a.cnt->max_ratio),
+              (unsigned long long)__double_as_longlong((double)__uint_as_float(s_mr)));
+}
+
 // --------------------------------------------------------------------------- correct
 template <typename T, int P, bool EXT>
 __global__ void correct_kernel(CheckArgs a, BoundParams bp, T *C) {
@@ -491,11 +554,6 @@ template <typename T, int P, bool EXT = false>
 aabft_status run_check(const aabft_config *cfg, const CheckArgs &a, BoundParams bp,
                        cudaStream_t st) {
   const int64_t nb = (cfg->M / cfg->bs) * (cfg->N / cfg->bs);
-  const size_t smem = (size_t)kCheckStrip * (cfg->bs + 1) * sizeof(double);
-  auto kern = check_kernel<T, P, EXT>;
-  if (smem > 48 * 1024) {
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  }
   if (nb > 0) {
     if (a.Rcol && a.Rrow) {
       // units of JB = 256/bs adjacent blocks of one block-row (bs <= 64 => JB >= 4)
@@ -504,8 +562,12 @@ aabft_status run_check(const aabft_config *cfg, const CheckArgs &a, BoundParams 
       const int64_t nunits = (cfg->M / cfg->bs) * ngrp;
       const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(nunits, 148 * 6));
       check_fused_kernel<T, P, EXT><<<grid, kFusedThreads, 0, st>>>(a, bp, nunits, (int)ngrp);
+    } else if (cfg->bs <= 128) {
+      dim3 grid((unsigned)((cfg->N + 127) / 128), (unsigned)(cfg->M / cfg->bs));
+      check_stream_kernel<T, P, EXT, 128><<<grid, 128, 0, st>>>(a, bp);
     } else {
-      kern<<<(unsigned)nb, kCheckThreads, smem, st>>>(a, bp);
+      dim3 grid((unsigned)((cfg->N + 255) / 256), (unsigned)(cfg->M / cfg->bs));
+      check_stream_kernel<T, P, EXT, 256><<<grid, 256, 0, st>>>(a, bp);
     }
     next_launch();
   }
