@@ -41,6 +41,12 @@ namespace {
 #define AABFT_F64_GROUP_M 16
 #endif
 constexpr int TILE = 64, BK = 16, STAGES = AABFT_F64_STAGES;
+// B tiles as 4 TMA boxes of 16 columns x 16 k with the 128B swizzle (B16) instead of 8 boxes of
+// 8 columns with the 64B swizzle: half the copies per stage; needs its own k-permutation
+#ifndef AABFT_F64_B16
+#define AABFT_F64_B16 0
+#endif
+constexpr bool B16 = AABFT_F64_B16 != 0;
 #ifndef AABFT_F64_NT
 #define AABFT_F64_NT 4
 #endif
@@ -213,7 +219,10 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
       const int k = kt * BK;
       if (lane == 0) mbar_arrive_expect_tx(&full[s], STAGE_BYTES);
       __syncwarp();
-      if (lane < 8) {
+      if (B16 && lane < 4) {
+        tma_load_2d(sa + A_BYTES + lane * 2048, tl.type == 2 ? &tmBcs : &tmB, &full[s],
+                    tl.n0 + lane * 16, k);
+      } else if (!B16 && lane < 8) {
         tma_load_2d(sa + A_BYTES + lane * 1024, tl.type == 2 ? &tmBcs : &tmB, &full[s],
                     tl.n0 + lane * 8, k);
       } else if (lane == 8) {
@@ -230,12 +239,24 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
   // With the 128B-swizzled A tile and the 64B-swizzled B boxes every half-warp of a 64-bit
   // LDS touches 16 distinct 8-byte bank slots (conflict-free: 2 wavefronts).
   // (offsets recomputed per load: cheaper than holding 8 registers across the k-loop)
+  // B16: k = pi16(ks, tig) from {0,3,12,15}, {1,2,13,14}, {4,7,8,11}, {5,6,9,10}: per k4-step
+  // the four tig give distinct (k>>3, k&1) -- conflict-free 128B-swizzled A rows -- and
+  // distinct (k>>1)&3 -- conflict-free 128B-swizzled 16-column B rows.
+  auto kperm = [&](int ks) -> int {
+    if (B16) {
+      constexpr uint64_t tab = 0xA965B874ED21FC30ull;  // nibble 4*ks + tig
+      return (int)((tab >> (4 * (4 * ks + tig))) & 15);
+    }
+    return (tig & 1) | ((ks & 1) << 1) | ((((tig >> 1) ^ (ks >> 1)) & 1) << 2) | ((tig >> 1) << 3);
+  };
   auto offA = [&](int ks) -> uint32_t {
-    const int k = (tig & 1) | ((ks & 1) << 1) | ((((tig >> 1) ^ (ks >> 1)) & 1) << 2) | ((tig >> 1) << 3);
+    const int k = kperm(ks);
     return (uint32_t)(((wm * 32 + g) * 16 + ((((k >> 1) ^ g) << 1) | (k & 1))) * 8);
   };
   auto offB = [&](int ks) -> uint32_t {
-    const int k = (tig & 1) | ((ks & 1) << 1) | ((((tig >> 1) ^ (ks >> 1)) & 1) << 2) | ((tig >> 1) << 3);
+    const int k = kperm(ks);
+    if (B16)  // nt-independent part; odd nt flips chunk bit 2 (see load)
+      return (uint32_t)(A_BYTES + wn * (WTN / 16) * 2048 + k * 128 + ((((g >> 1) ^ (k & 7)) << 4) | ((g & 1) << 3)));
     return (uint32_t)(A_BYTES + wn * NT * 1024 + (k * 8 + ((((g >> 1) ^ ((k >> 1) & 3)) << 1) | (g & 1))) * 8);
   };
 
@@ -294,9 +315,16 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
         a[buf][mt][0] = *reinterpret_cast<const double *>(st + offA(ks) + mt * 2048);
         a[buf][mt][1] = *reinterpret_cast<const double *>(st + offA(ks) + mt * 2048 + 1024);
       }
+      if (B16) {
+        const uint32_t ob = offB(ks);
 #pragma unroll
-      for (int nt = 0; nt < NT; ++nt)
-        b[buf][nt] = *reinterpret_cast<const double *>(st + offB(ks) + nt * 1024);
+        for (int nt = 0; nt < NT; ++nt)
+          b[buf][nt] = *reinterpret_cast<const double *>(st + ((ob + (nt >> 1) * 2048) ^ ((nt & 1) << 6)));
+      } else {
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt)
+          b[buf][nt] = *reinterpret_cast<const double *>(st + offB(ks) + nt * 1024);
+      }
     };
     {
       const int s0 = j % STAGES;
@@ -637,14 +665,17 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
 
   CUtensorMap tA, tAcs, tB, tBcs;
   if (!make_map(&tA, A, K, M, lda, BK, TILE, CU_TENSOR_MAP_SWIZZLE_128B)) return AABFT_EINVAL;
-  if (!make_map(&tB, B, N, K, ldb, 8, BK, CU_TENSOR_MAP_SWIZZLE_64B)) return AABFT_EINVAL;
+  if (!make_map(&tB, B, N, K, ldb, B16 ? 16 : 8, BK,
+                B16 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B))
+    return AABFT_EINVAL;
   if (plain) {
     tAcs = tA;
     tBcs = tB;
   } else {
     if (!make_map(&tAcs, enc->Acs, K, a.Mcs, enc->ld_acs, BK, TILE, CU_TENSOR_MAP_SWIZZLE_128B))
       return AABFT_EINVAL;
-    if (!make_map(&tBcs, enc->Bcs, a.Ncs, K, enc->ld_bcs, 8, BK, CU_TENSOR_MAP_SWIZZLE_64B))
+    if (!make_map(&tBcs, enc->Bcs, a.Ncs, K, enc->ld_bcs, B16 ? 16 : 8, BK,
+                  B16 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B))
       return AABFT_EINVAL;
   }
   if (total > 0) {
