@@ -310,6 +310,22 @@ class ProtectedGemm:
             self.correct(stream)
         return self.result()
 
+    def capture(self, A, B, *, correct: bool = True):
+        """Record encode -> gemm -> check -> correct for these (fixed) A, B buffers as one CUDA
+        graph; ``graph.replay()`` re-runs the whole protected product (new contents of A and B
+        are picked up).  For launch-latency-bound sizes (BASELINE configs[0]: 128^3 is ~10 us
+        of GPU work against ~8 launches).  The first eager run sets the kernels' one-time
+        attributes outside the capture."""
+        side = torch.cuda.Stream(self.device)
+        side.wait_stream(torch.cuda.current_stream(self.device))
+        with torch.cuda.stream(side):
+            self.run(A, B, correct=correct)
+        torch.cuda.current_stream(self.device).wait_stream(side)
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph):
+            self.run(A, B, correct=correct)
+        return graph
+
     def result(self) -> Result:
         return Result(self.C, self.Ccol, self.Crow, self.Acs, self.Bcs, self.topA_val,
                       self.topA_idx, self.topB_val, self.topB_idx, self.reports, self.counts,

@@ -552,3 +552,30 @@ def test_gpu_bound_column_tables(P, orc, n, table):
     m = float(torch.cat([b["eps_col"].ravel(), b["eps_row"].ravel()]).mean())
     paper = g["rows"][str(n)]["avg_aabft"]
     assert 0.95 * paper <= m <= 1.05 * paper, (m, paper)
+
+
+@pytest.mark.parametrize("dtype", [np.float64, np.float32])
+def test_cuda_graph_replay(P, orc, dtype):
+    """The four C-ABI calls captured in one CUDA graph: a replay equals the eager run bit for
+    bit, and picks up new contents of the captured input buffers."""
+    M = N = K = 128
+    bs, p = 32, 2
+    A = gen("uniform", M, K, 31, 0, dtype)
+    B = gen("uniform", K, N, 31, 1, dtype)
+    dA, dB = to_dev(A), to_dev(B)
+    plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p)
+    g = plan.capture(dA, dB)
+    g.replay()
+    torch.cuda.synchronize()
+    C1, cnt1 = host(plan.C).copy(), plan.result().counts()
+    eager = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p)
+    res = eager.run(dA, dB)
+    torch.cuda.synchronize()
+    assert np.array_equal(C1, host(res.C)) and cnt1 == res.counts()
+    A2 = gen("uniform", M, K, 32, 0, dtype)
+    dA.copy_(torch.from_numpy(A2).cuda())
+    g.replay()
+    torch.cuda.synchronize()
+    o = orc.protected_matmul(A2, B, bs=bs, p=p)
+    assert norm_err(host(plan.C), o["C"], A2, B) <= (1e-13 if dtype == np.float64 else 0.0)
+    assert plan.result().counts()["clean"] == (M // bs) * (N // bs)
