@@ -71,12 +71,17 @@ __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, 
     int ix[P];
     tp_init<P>(v, ix);
     if (r < rows) {
+      // ascending columns into this lane's own list: the new element loses every tie.  The
+      // column limit is hoisted (32-bit: K < 2^31 is validated) so the scan carries no
+      // per-element guard or 64-bit index arithmetic.
+      const int kbase = chunk * kEncAChunk;
+      const int lim = K - kbase < kEncAChunk ? (int)(K - kbase) : kEncAChunk;
+      const double *trow = tile[r];
+      // (measured: a fully or 8x unrolled version of this loop returned a list holding one
+      // element twice on sm_100a; 4x with the compile-time bound is parity-clean)
 #pragma unroll 4
-      for (int cc = q; cc < kEncAChunk; cc += 4) {
-        const int64_t kk = (int64_t)chunk * kEncAChunk + cc;
-        // ascending columns into this lane's own list: the new element loses every tie
-        if (kk < K) tp_push<P>(v, ix, tile[r][cc], (int)kk);
-      }
+      for (int cc = q; cc < kEncAChunk; cc += 4)
+        if (cc < lim) tp_push<P>(v, ix, trow[cc], kbase + cc);
     }
     tp_shfl_merge<P>(v, ix, 1);
     tp_shfl_merge<P>(v, ix, 2);
@@ -157,13 +162,20 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
   if (kbeg < kend) load_strip(kbeg);
   for (int64_t k0 = kbeg; k0 < kend; k0 += SB) {
     const int rows = (int)(kend - k0 < SB ? kend - k0 : SB);
+    const int k0i = (int)k0;  // K < 2^31 (validated)
+    if (rows == SB) {  // full strip: no per-element guard
 #pragma unroll
-    for (int rr = 0; rr < SB; ++rr) {
-      if (rr < rows) {
+      for (int rr = 0; rr < SB; ++rr) {
         tile[rr][c] = vals[rr];
-        if (TOPP && jin) {  // ascending k, own list: the new element loses every tie
-          const double a = fabs((double)vals[rr]);
-          tp_push<P>(v, ix, a, (int)(k0 + rr));
+        // ascending k, own list: the new element loses every tie
+        if (TOPP && jin) tp_push<P>(v, ix, fabs((double)vals[rr]), k0i + rr);
+      }
+    } else {
+#pragma unroll
+      for (int rr = 0; rr < SB; ++rr) {
+        if (rr < rows) {
+          tile[rr][c] = vals[rr];
+          if (TOPP && jin) tp_push<P>(v, ix, fabs((double)vals[rr]), k0i + rr);
         }
       }
     }
