@@ -80,8 +80,14 @@ SHAPES = [
 ]
 
 
+ENCODE_SHAPES = SHAPES + [
+    (512, 768, 2048, 64, 2),   # many 128-column chunks of A, several k-chunks of B, p = 2
+    (256, 256, 4099, 32, 3),   # ragged last chunk with an odd K
+]
+
+
 @pytest.mark.parametrize("dtype", [np.float64, np.float32])
-@pytest.mark.parametrize("shape", SHAPES)
+@pytest.mark.parametrize("shape", ENCODE_SHAPES)
 def test_encode_bit_exact(P, orc, dtype, shape):
     M, N, K, bs, p = shape
     A = gen("uniform", M, K, 3, 0, dtype)
