@@ -1,5 +1,6 @@
 // api.cu -- the C ABI of include/aabft.h: validation, workspace sizing, dispatch, errors.
 // No C++ exception crosses the ABI; every entry point is stream-ordered and never allocates.
+#include <cstdlib>
 #include <algorithm>
 #include <atomic>
 #include <cmath>
@@ -382,6 +383,7 @@ aabft_status aabft_correct_ext(const aabft_config *cfg, const aabft_product *pro
 // A_i and B_j have landed (encode of a slab / panel runs once), and each finished C block is
 // copied back on a third stream -- PCIe in both directions overlaps the DMMA GEMMs.
 namespace {
+constexpr int kMaxSplit = 8, kDefaultSplit = 4;
 struct Split {
   int S;
   int64_t ms, ns;  // slab rows / panel cols (last may be shorter)
@@ -391,7 +393,14 @@ Split plan_split(const aabft_config *c) {
   // additionally keep the Bcs / Crow column offsets 16-byte aligned (4 x (N/bs) granules)
   const int64_t unit = std::max<int64_t>(64, c->bs), unit_n = 4 * unit;
   Split sp;
-  sp.S = (int)std::max<int64_t>(1, std::min<int64_t>(4, std::min(c->M / (4 * unit), c->N / unit_n)));
+  // S x S blocks: finer splits start the GEMMs earlier and leave less work after the last
+  // host->device copy, at the cost of smaller GEMM launches (AABFT_HOST_SPLIT overrides the cap)
+  static const int cap = [] {
+    const char *e = std::getenv("AABFT_HOST_SPLIT");
+    const int v = e ? std::atoi(e) : 0;
+    return v >= 1 && v <= kMaxSplit ? v : kDefaultSplit;
+  }();
+  sp.S = (int)std::max<int64_t>(1, std::min<int64_t>(cap, std::min(c->M / (4 * unit), c->N / unit_n)));
   sp.ms = (c->M / sp.S + unit - 1) / unit * unit;
   sp.ns = (c->N / sp.S + unit_n - 1) / unit_n * unit_n;
   return sp;
@@ -438,7 +447,7 @@ Arena plan_arena(const aabft_config *c) {
 }
 struct HostPipe {  // per-device copy streams + event pool (created once; the library's runtime)
   cudaStream_t in = nullptr, out = nullptr;
-  cudaEvent_t ev[40];
+  cudaEvent_t ev[2 * kMaxSplit + kMaxSplit * kMaxSplit + 2];
   bool ok = false;
 };
 HostPipe &host_pipe() {
@@ -484,8 +493,9 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
   const int64_t M = cfg->M, N = cfg->N, K = cfg->K, bs = cfg->bs, p = cfg->p;
   const Split sp = plan_split(cfg);
   const int S = sp.S;
-  cudaEvent_t *evA = hp.ev, *evB = hp.ev + 4, *evC = hp.ev + 8;  // evC: S*S <= 16
-  cudaEvent_t evStart = hp.ev[24], evOutDone = hp.ev[25];
+  cudaEvent_t *evA = hp.ev, *evB = hp.ev + kMaxSplit, *evC = hp.ev + 2 * kMaxSplit;  // S*S
+  cudaEvent_t evStart = hp.ev[2 * kMaxSplit + kMaxSplit * kMaxSplit];
+  cudaEvent_t evOutDone = hp.ev[2 * kMaxSplit + kMaxSplit * kMaxSplit + 1];
   // the copy streams start after whatever the caller enqueued before this call
   if (cudaEventRecord(evStart, st) != cudaSuccess || cudaStreamWaitEvent(hp.in, evStart, 0) != cudaSuccess ||
       cudaStreamWaitEvent(hp.out, evStart, 0) != cudaSuccess)
@@ -512,7 +522,7 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
   auto tbv = [&](int j) { return reinterpret_cast<double *>(base + a.oTbv) + (j * sp.ns + j * (sp.ns / bs)) * p; };
   auto tbi = [&](int j) { return reinterpret_cast<int32_t *>(base + a.oTbi) + (j * sp.ns + j * (sp.ns / bs)) * p; };
   size_t rcol_off = 0, rrow_off = 0, rep_off = 0;
-  bool encA[4] = {false, false, false, false}, encB[4] = {false, false, false, false};
+  bool encA[kMaxSplit] = {}, encB[kMaxSplit] = {};
   int nblk = 0;
   // compute order: diagonal shells, so block (i, j) runs as soon as A_i and B_j are resident
   for (int d = 0; d < S; ++d) {
