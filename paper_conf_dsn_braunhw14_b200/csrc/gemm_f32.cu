@@ -14,6 +14,8 @@
 // k-tile replays that k-tile step by step in scalar code -- site 4 rounds the product on its
 // own and XORs it ("errorVecMul"), sites 1 / 3 hit the accumulator right after step k_step
 // ("errorVecAdd1") -- so a faulty FP32 product equals the oracle's dot_fault bit for bit.
+#include <atomic>
+
 #include "common.cuh"
 
 namespace aabft {
@@ -329,12 +331,14 @@ aabft_status launch_gemm_f32(const aabft_config *cfg, const void *A, int64_t lda
   a.faults = faults;
   a.nfaults = faults ? nfaults : 0;
   const int64_t tiles = a.n0 + a.n1 + a.n2;
-  static bool attr = false;
-  if (!attr) {
+  static std::atomic<bool> attr_dev[64];  // per device (function attributes are per context)
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (!attr_dev[dev & 63].load(std::memory_order_relaxed)) {
     if (cudaFuncSetAttribute(gemm_f32_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM32) != cudaSuccess ||
         cudaFuncSetAttribute(gemm_f32_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM32) != cudaSuccess)
       return check_launch("gemm_f32 smem attribute");
-    attr = true;
+    attr_dev[dev & 63].store(true, std::memory_order_relaxed);
   }
   if (tiles > 0) {
     if (a.nfaults > 0) gemm_f32_kernel<true><<<(unsigned)tiles, THREADS, SMEM32, st>>>(a);

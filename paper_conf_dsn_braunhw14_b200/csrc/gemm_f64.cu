@@ -27,6 +27,7 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <atomic>
 
 #include "common.cuh"
 
@@ -608,10 +609,14 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
                              int64_t ldb, const aabft_encoded *enc, const aabft_product *out,
                              const aabft_fault *faults, int32_t nfaults, bool plain, void *ws,
                              cudaStream_t st) {
-  static int max_ctas = 0;
+  // per-device one-time setup (function attributes belong to the device's context); a racing
+  // first call computes the same value twice, which is benign
+  static std::atomic<int> max_ctas_dev[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int max_ctas = max_ctas_dev[dev & 63].load(std::memory_order_relaxed);
   if (!max_ctas) {
-    int dev = 0, sms = 0, per_sm = 0;
-    cudaGetDevice(&dev);
+    int sms = 0, per_sm = 0;
     if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
       return check_launch("gemm_f64 SM count");
     if (cudaFuncSetAttribute(gemm_f64_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -622,6 +627,7 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
       return check_launch("gemm_f64 occupancy");
     // every CTA must be resident (split-tile owners wait on later CTAs)
     max_ctas = std::min(sms * per_sm, kMaxCtas);
+    max_ctas_dev[dev & 63].store(max_ctas, std::memory_order_relaxed);
   }
   const int64_t M = cfg->M, N = cfg->N, K = cfg->K, bs = cfg->bs;
   GemmArgs a{};
