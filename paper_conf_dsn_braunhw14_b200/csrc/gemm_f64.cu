@@ -48,6 +48,9 @@ constexpr int TILE = 64, BK = 16, STAGES = AABFT_F64_STAGES;
 #define AABFT_F64_B16 0
 #endif
 constexpr bool B16 = AABFT_F64_B16 != 0;
+#ifndef AABFT_F64_L2PROMO
+#define AABFT_F64_L2PROMO CU_TENSOR_MAP_L2_PROMOTION_L2_128B
+#endif
 #ifndef AABFT_F64_NT
 #define AABFT_F64_NT 4
 #endif
@@ -574,7 +577,7 @@ bool make_map(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer, 
   cuuint32_t box[2] = {box_inner, box_outer};
   cuuint32_t es[2] = {1, 1};
   CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 2, const_cast<void *>(base), dims, strides,
-                   box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                   box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, sw, AABFT_F64_L2PROMO,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     set_error("cuTensorMapEncodeTiled failed (%d): inner=%llu outer=%llu ld=%llu", (int)r,
