@@ -34,7 +34,10 @@ BoundParams make_bound_params(const aabft_config *cfg);
 
 // Encode-stage chunking (shared by workspace sizing and the launcher).
 constexpr int kEncAChunk = 128;   // columns of A per encode CTA (one thread per column)
-constexpr int kEncBChunk = 256;   // rows of B per encode CTA
+#ifndef AABFT_ENC_BCHUNK
+#define AABFT_ENC_BCHUNK 256
+#endif
+constexpr int kEncBChunk = AABFT_ENC_BCHUNK;  // rows of B per encode CTA
 inline int64_t enc_a_chunks(int64_t K) { return (K + kEncAChunk - 1) / kEncAChunk; }
 inline int64_t enc_b_chunks(int64_t K) { return (K + kEncBChunk - 1) / kEncBChunk; }
 
