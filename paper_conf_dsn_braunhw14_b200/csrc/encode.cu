@@ -11,6 +11,9 @@
 // (running top-p over k in registers) and the BS-wide row sums are taken from the staged
 // tile, one sequential thread per (row, block).  Partial top-p lists per chunk are reduced
 // by a warp-per-vector kernel that also computes the top-p of the checksum vectors.
+// Strips are double-buffered in registers (the next strip's loads are in flight during the
+// top-p / row-sum phase) and the top-p insertion is branch-free for p <= 4 (tp_push), so a
+// warp never diverges on inserts: 44 + 43 + 9 us at 4096^2 FP64.
 #include <algorithm>
 
 #include "common.cuh"
