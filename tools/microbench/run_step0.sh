@@ -4,7 +4,8 @@ set -x
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv
 nvidia-smi --query-gpu=index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active --format=csv -lms 200 > gpurun_out/step0_clocks.csv &
 SMI=$!
-./tools/microbench/fp64_pipes | tee gpurun_out/step0_pipes.jsonl
+nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o /tmp/fp64_pipes tools/microbench/fp64_pipes.cu
+/tmp/fp64_pipes | tee gpurun_out/step0_pipes.jsonl
 python - <<'PY' | tee gpurun_out/step0_cublas.jsonl
 import torch, json, time
 for dt, n in [(torch.float64, 4096), (torch.float64, 8192), (torch.float32, 8192)]:
