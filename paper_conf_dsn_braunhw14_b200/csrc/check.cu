@@ -250,61 +250,71 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
       s_rmax[tid] = 0u;
     }
     __syncthreads();
-    // ---- column check (I, j): Rcol (+ the epilogue's second part) vs carried Ccol[I][j]
+    // Both checks' operands are gathered first (every load of the thread in flight together),
+    // then the part sums are written back, then classified.
+    const int Jc = tid / bs;                                   // column check: block of j
+    const int64_t j = J0 * bs + tid;
+    const int ii = tid / JB, Jr = tid - (tid / JB) * JB;      // row check: (i, J)
+    const int64_t J = J0 + Jr, i = I * bs + ii;
+    const bool hc = j < a.N, hr = J < nJ;
+    double refc = 0.0, carc = 0.0, refr = 0.0, carr = 0.0, rc2 = 0.0, rp[7] = {};  // row_parts <= 64 / 8
+    Bound bc{0.0, 0.0}, brw{0.0, 0.0};
+    if (hc) {  // column check (I, j): Rcol (+ the epilogue's second part) vs carried Ccol[I][j]
+      refc = a.Rcol[I * a.N + j];
+      if (a.col_parts > 1) rc2 = a.Rcol2[I * a.N + j];
+      carc = (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
+      bc = col_bound<EXT, P>(a, bp, I, j);
+    }
+    if (hr) {  // row check (i, J): Rrow (+ parts) vs carried Crow[i][J]
+      refr = a.Rrow[i * nJ + J];
+      for (int q = 1; q < a.row_parts && q <= 7; ++q)
+        rp[q - 1] = a.Rrow2[(q - 1) * a.M * nJ + i * nJ + J];
+      carr = (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
+      brw = row_bound<EXT, P>(a, bp, i, J);
+    }
+    // complete the epilogue parts in their fixed order and leave the full sums in Rcol / Rrow;
+    // the consumed parts are zeroed so a second check (another bound) sees the same sums
+    if (hc && a.col_parts > 1) {
+      refc = refc + rc2;
+      const_cast<double *>(a.Rcol)[I * a.N + j] = refc;
+      const_cast<double *>(a.Rcol2)[I * a.N + j] = 0.0;
+    }
+    if (hr && a.row_parts > 1) {
+      for (int q = 1; q < a.row_parts && q <= 7; ++q) {
+        refr = refr + rp[q - 1];
+        const_cast<double *>(a.Rrow2)[(q - 1) * a.M * nJ + i * nJ + J] = 0.0;
+      }
+      const_cast<double *>(a.Rrow)[i * nJ + J] = refr;
+    }
     {
-      const int Jl = tid / bs;
-      const int64_t j = J0 * bs + tid;
       float r = 0.f;
-      if (j < a.N) {
-        double *rc = const_cast<double *>(a.Rcol) + I * a.N + j;
-        double ref = *rc;
-        if (a.col_parts > 1) {  // complete the parts and leave the full sum in Rcol; the
-          double *rc2 = const_cast<double *>(a.Rcol2) + I * a.N + j;  // consumed part is zeroed
-          ref = ref + *rc2;  // so a second check (another bound) sees the same sums
-          *rc = ref;
-          *rc2 = 0.0;
-        }
-        const double d = ref - (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
-        const Bound b = col_bound<EXT, P>(a, bp, I, j);
-        const int cl = classify(d, b);
+      if (hc) {
+        const double d = refc - carc;
+        const int cl = classify(d, bc);
         cls_tot[cl] += 1;
         if (cl) {
-          atomicMax(&s_worst[Jl], cl);
-          if (cl == 2) { atomicAdd(&s_nc[Jl], 1); s_col[Jl] = (int)j; }
+          atomicMax(&s_worst[Jc], cl);
+          if (cl == 2) { atomicAdd(&s_nc[Jc], 1); s_col[Jc] = (int)j; }
         }
-        r = (float)ratio_fast(d, b.eps);
+        r = (float)ratio_fast(d, bc.eps);
       }
       for (int m = 1; m < cseg; m <<= 1) r = fmaxf(r, __shfl_xor_sync(0xffffffffu, r, m));
-      if ((lane & (cseg - 1)) == 0 && r > 0.f) atomicMax(&s_rmax[Jl], __float_as_uint(r));
+      if ((lane & (cseg - 1)) == 0 && r > 0.f) atomicMax(&s_rmax[Jc], __float_as_uint(r));
     }
-    // ---- row check (i, J): Rrow (+ parts) vs carried Crow[i][J]
     {
-      const int ii = tid / JB, Jl = tid - (tid / JB) * JB;
-      const int64_t J = J0 + Jl, i = I * bs + ii;
       float r = 0.f;
-      if (J < nJ) {
-        double *rr = const_cast<double *>(a.Rrow) + i * nJ + J;
-        double ref = *rr;
-        if (a.row_parts > 1) {
-          for (int q = 1; q < a.row_parts; ++q) {
-            double *part = const_cast<double *>(a.Rrow2) + (q - 1) * a.M * nJ + i * nJ + J;
-            ref = ref + *part;
-            *part = 0.0;
-          }
-          *rr = ref;
-        }
-        const double d = ref - (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
-        const Bound b = row_bound<EXT, P>(a, bp, i, J);
-        const int cl = classify(d, b);
+      if (hr) {
+        const double d = refr - carr;
+        const int cl = classify(d, brw);
         cls_tot[cl] += 1;
         if (cl) {
-          atomicMax(&s_worst[Jl], cl);
-          if (cl == 2) { atomicAdd(&s_nr[Jl], 1); s_row[Jl] = (int)i; }
+          atomicMax(&s_worst[Jr], cl);
+          if (cl == 2) { atomicAdd(&s_nr[Jr], 1); s_row[Jr] = (int)i; }
         }
-        r = (float)ratio_fast(d, b.eps);
+        r = (float)ratio_fast(d, brw.eps);
       }
       for (int m = JB; m < 32; m <<= 1) r = fmaxf(r, __shfl_xor_sync(0xffffffffu, r, m));
-      if (lane < JB && r > 0.f) atomicMax(&s_rmax[Jl], __float_as_uint(r));
+      if (lane < JB && r > 0.f) atomicMax(&s_rmax[Jr], __float_as_uint(r));
     }
     __syncthreads();
     // ---- block verdicts (warp 0: JB <= 32 blocks)
