@@ -165,6 +165,9 @@ __device__ __forceinline__ double xor_bits(double v, uint64_t m) {
   return __longlong_as_double(__double_as_longlong(v) ^ (long long)m);
 }
 
+// FAULTS: the Alg 3 injection instantiation (launched only with a fault list); the production
+// instantiation carries no fault bookkeeping in its k-loop.
+template <bool FAULTS>
 __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
     gemm_f64_kernel(const __grid_constant__ CUtensorMap tmA,
                     const __grid_constant__ CUtensorMap tmAcs,
@@ -277,7 +280,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
 
     // faults that hit this tile (output coordinates of the tile's product)
     int nf = 0;
-    if (args.nfaults > 0) {
+    if (FAULTS && args.nfaults > 0) {
       mma_sync_bar();
       if (threadIdx.x == 0) *s_nf = 0;
       mma_sync_bar();
@@ -356,7 +359,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
       // release the stage to the producer (its last fragments were consumed by the ks = 3 DMMAs)
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[s]);
-      if (nf > 0) {  // Alg 3 errorVecAdd1 at k-tile granularity
+      if (FAULTS && nf > 0) {  // Alg 3 errorVecAdd1 at k-tile granularity
         for (int f = 0; f < nf; ++f) {
           const aabft_fault ft = s_f[f];
           if ((ft.site != 1 && ft.site != 3) || ft.k_step / BK != kt) continue;
@@ -414,7 +417,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
         mma_sync_bar();
       }
     }
-    if (nf > 0) {
+    if (FAULTS && nf > 0) {
       for (int f = 0; f < nf; ++f) {
         const aabft_fault ft = s_f[f];
         if (ft.site != 0 && ft.site != 2) continue;
@@ -622,14 +625,20 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
     int sms = 0, per_sm = 0;
     if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
       return check_launch("gemm_f64 SM count");
-    if (cudaFuncSetAttribute(gemm_f64_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    if (cudaFuncSetAttribute(gemm_f64_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             SMEM_BYTES) != cudaSuccess ||
+        cudaFuncSetAttribute(gemm_f64_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              SMEM_BYTES) != cudaSuccess)
       return check_launch("gemm_f64 smem attribute");
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, gemm_f64_kernel, CTA_THREADS,
+    int per_sm_f = 0;  // both instantiations must keep every CTA resident
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm_f, gemm_f64_kernel<true>, CTA_THREADS,
+                                                      SMEM_BYTES) != cudaSuccess)
+      return check_launch("gemm_f64 occupancy");
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, gemm_f64_kernel<false>, CTA_THREADS,
                                                       SMEM_BYTES) != cudaSuccess || per_sm < 1)
       return check_launch("gemm_f64 occupancy");
     // every CTA must be resident (split-tile owners wait on later CTAs)
-    max_ctas = std::min(sms * per_sm, kMaxCtas);
+    max_ctas = std::min(sms * std::min(per_sm, per_sm_f), kMaxCtas);
     max_ctas_dev[dev & 63].store(max_ctas, std::memory_order_relaxed);
   }
   const int64_t M = cfg->M, N = cfg->N, K = cfg->K, bs = cfg->bs;
@@ -690,7 +699,10 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
   if (total > 0) {
     if (a.sk_iters > 0 && cudaMemsetAsync(a.flags, 0, kMaxCtas * sizeof(int), st) != cudaSuccess)
       return check_launch("gemm_f64 flag reset");
-    gemm_f64_kernel<<<grid, CTA_THREADS, SMEM_BYTES, st>>>(tA, tAcs, tB, tBcs, a);
+    if (a.nfaults > 0)
+      gemm_f64_kernel<true><<<grid, CTA_THREADS, SMEM_BYTES, st>>>(tA, tAcs, tB, tBcs, a);
+    else
+      gemm_f64_kernel<false><<<grid, CTA_THREADS, SMEM_BYTES, st>>>(tA, tAcs, tB, tBcs, a);
     next_launch();
   }
   return check_launch("aabft_gemm(f64)");
