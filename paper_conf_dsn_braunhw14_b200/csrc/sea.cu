@@ -11,9 +11,9 @@
 //
 // Work: the norms read A, B (and the small Acs, Bcs) once: M*K + K*N elements, HBM-bound in
 // principle but each norm is one sequential dependency chain of K double adds (the paper's
-// "vector norms use only a small fraction of the available GPU threads").  Rows are
-// one thread each with 16-byte vector loads (each thread's row stays in L1 across its
-// iterations); columns are one thread each with coalesced row-segment loads.
+// "vector norms use only a small fraction of the available GPU threads").  The chain
+// stays one thread per vector; the loads feeding it are spread over 256-thread CTAs of 16
+// vectors each (sea_norm_kernel), so the ~260 CTAs cover every SM with 32 KiB in flight.
 #include <algorithm>
 
 #include "common.cuh"
@@ -21,70 +21,72 @@
 namespace aabft {
 namespace {
 
-// ||row r||_2 for R rows of an R x L row-major matrix (two matrices per launch: A then Acs)
-template <typename T>
-__global__ void __launch_bounds__(128) sea_norm_rows_kernel(const T *__restrict__ X0, int64_t ld0,
-                                                            int64_t R0, const T *__restrict__ X1,
-                                                            int64_t ld1, int64_t R1, int64_t L,
-                                                            double *__restrict__ out) {
-  const int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (r >= R0 + R1) return;
-  const T *x = r < R0 ? X0 + r * ld0 : X1 + (r - R0) * ld1;
-  double s = 0.0;
-  constexpr int V = 16 / sizeof(T);  // elements per 16-byte load (rows are 16-B aligned)
-  int64_t k = 0;
-  for (; k + 4 * V <= L; k += 4 * V) {
-    T v[4 * V];
+// ||x||_2 of R0 + R1 vectors of length L, 16 vectors per 256-thread CTA.  ROWS: vector r is
+// row r of a row-major matrix (X0 for r < R0, then X1); else vector c is column c.  The CTA
+// stages a 16 x 128 tile of the vectors in shared memory with coalesced loads from all 8 warps
+// (ROWS: a warp reads 32 consecutive k of one row; columns: a half-warp reads 16 consecutive
+// columns of one k-row), the next tile's loads are in flight in registers while lanes 0..15 of
+// warp 0 add their vector's 128 squares in ascending k -- the sequential chain of the
+// definition, bit-identical to the oracle (zero padding past L adds +0 to a sum >= 0, exact).
+constexpr int kSeaVec = 16, kSeaTile = 128, kSeaThreads = 256;
+constexpr int kSeaPer = kSeaVec * kSeaTile / kSeaThreads;  // elements per thread per tile
+
+template <typename T, bool ROWS>
+__global__ void __launch_bounds__(kSeaThreads) sea_norm_kernel(const T *__restrict__ X0,
+                                                               int64_t ld0, int64_t R0,
+                                                               const T *__restrict__ X1,
+                                                               int64_t ld1, int64_t R1, int64_t L,
+                                                               double *__restrict__ out) {
+  __shared__ double tile[2][kSeaVec][kSeaTile + 1];  // stride 129: conflict-free per-vector reads
+  const int t = threadIdx.x;
+  const int64_t v0 = (int64_t)blockIdx.x * kSeaVec;
+  // this thread's kSeaPer (vector, k) slots of a tile and the base pointer of each
+  const T *base[kSeaPer];
+  int64_t step[kSeaPer];  // element stride along k
+  int sv[kSeaPer], sk[kSeaPer];
+  bool ok[kSeaPer];
 #pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      if constexpr (V == 2) {
-        const double2 q = __ldg(reinterpret_cast<const double2 *>(x + k) + u);
-        v[u * V] = (T)q.x; v[u * V + 1] = (T)q.y;
-      } else {
-        const float4 q = __ldg(reinterpret_cast<const float4 *>(x + k) + u);
-        v[u * V] = (T)q.x; v[u * V + 1] = (T)q.y; v[u * V + 2] = (T)q.z; v[u * V + 3] = (T)q.w;
+  for (int e = 0; e < kSeaPer; ++e) {
+    const int idx = t + kSeaThreads * e;
+    sv[e] = ROWS ? idx / kSeaTile : idx % kSeaVec;
+    sk[e] = ROWS ? idx % kSeaTile : idx / kSeaVec;
+    const int64_t v = v0 + sv[e];
+    ok[e] = v < R0 + R1;
+    const bool first = v < R0;
+    if (ROWS) {
+      base[e] = ok[e] ? (first ? X0 + v * ld0 : X1 + (v - R0) * ld1) : X0;
+      step[e] = 1;
+    } else {
+      base[e] = ok[e] ? (first ? X0 + v : X1 + (v - R0)) : X0;
+      step[e] = first ? ld0 : ld1;
+    }
+  }
+  double regs[kSeaPer];
+  auto load = [&](int64_t k0) {
+#pragma unroll
+    for (int e = 0; e < kSeaPer; ++e) {
+      const int64_t k = k0 + sk[e];
+      regs[e] = (ok[e] && k < L) ? (double)__ldg(base[e] + k * step[e]) : 0.0;
+    }
+  };
+  const int nt = (int)((L + kSeaTile - 1) / kSeaTile);
+  double s = 0.0;
+  load(0);
+  for (int it = 0; it < nt; ++it) {
+    double(*buf)[kSeaTile + 1] = tile[it & 1];
+#pragma unroll
+    for (int e = 0; e < kSeaPer; ++e) buf[sv[e]][sk[e]] = regs[e];
+    __syncthreads();  // also orders warp 0's reads of tile[it & 1] two tiles ago before this store
+    if (it + 1 < nt) load((int64_t)(it + 1) * kSeaTile);
+    if (t < kSeaVec) {
+#pragma unroll 16
+      for (int k = 0; k < kSeaTile; ++k) {
+        const double d = buf[t][k];
+        s = __dadd_rn(s, __dmul_rn(d, d));  // ascending k
       }
     }
-#pragma unroll
-    for (int e = 0; e < 4 * V; ++e) {
-      const double d = (double)v[e];
-      s = __dadd_rn(s, __dmul_rn(d, d));  // ascending k
-    }
   }
-  for (; k < L; ++k) {
-    const double d = (double)__ldg(x + k);
-    s = __dadd_rn(s, __dmul_rn(d, d));
-  }
-  out[r] = __dsqrt_rn(s);
-}
-
-// ||column c||_2 for the C0 columns of X0 (L x C0) then the C1 columns of X1 (L x C1)
-template <typename T>
-__global__ void __launch_bounds__(128) sea_norm_cols_kernel(const T *__restrict__ X0, int64_t ld0,
-                                                            int64_t C0, const T *__restrict__ X1,
-                                                            int64_t ld1, int64_t C1, int64_t L,
-                                                            double *__restrict__ out) {
-  const int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  if (c >= C0 + C1) return;
-  const T *x = c < C0 ? X0 + c : X1 + (c - C0);
-  const int64_t ld = c < C0 ? ld0 : ld1;
-  double s = 0.0;
-  int64_t k = 0;
-  for (; k + 8 <= L; k += 8) {
-    T v[8];
-#pragma unroll
-    for (int u = 0; u < 8; ++u) v[u] = __ldg(x + (k + u) * ld);
-#pragma unroll
-    for (int u = 0; u < 8; ++u) {
-      const double d = (double)v[u];
-      s = __dadd_rn(s, __dmul_rn(d, d));
-    }
-  }
-  for (; k < L; ++k) {
-    const double d = (double)__ldg(x + k * ld);
-    s = __dadd_rn(s, __dmul_rn(d, d));
-  }
-  out[c] = __dsqrt_rn(s);
+  if (t < kSeaVec && v0 + t < R0 + R1) out[v0 + t] = __dsqrt_rn(s);
 }
 
 // SA[I] = sum of the bs row norms of block-row I, SB[J] likewise (sequential ascending)
@@ -142,9 +144,9 @@ aabft_status run_sea(const aabft_config *cfg, const T *A, int64_t lda, const T *
   double *nB = nA + (M + nI);               // N + nJ: columns of B, then columns of Bcs
   double *SA = nB + (N + nJ);
   double *SB = SA + nI;
-  sea_norm_rows_kernel<T><<<(unsigned)((M + nI + 127) / 128), 128, 0, st>>>(
+  sea_norm_kernel<T, true><<<(unsigned)((M + nI + kSeaVec - 1) / kSeaVec), kSeaThreads, 0, st>>>(
       A, lda, M, static_cast<const T *>(enc->Acs), enc->ld_acs, nI, K, nA);
-  sea_norm_cols_kernel<T><<<(unsigned)((N + nJ + 127) / 128), 128, 0, st>>>(
+  sea_norm_kernel<T, false><<<(unsigned)((N + nJ + kSeaVec - 1) / kSeaVec), kSeaThreads, 0, st>>>(
       B, ldb, N, static_cast<const T *>(enc->Bcs), enc->ld_bcs, nJ, K, nB);
   sea_block_sums_kernel<<<(unsigned)((nI + nJ + 127) / 128), 128, 0, st>>>(nA, nI, nB, nJ,
                                                                            (int)bs, SA, SB);
