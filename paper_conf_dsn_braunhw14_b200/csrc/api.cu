@@ -379,8 +379,9 @@ aabft_status aabft_correct_ext(const aabft_config *cfg, const aabft_product *pro
 // Pipelined: A is split into S row slabs and B into S column panels (S <= 4, multiples of
 // lcm(bs, 64)); the S x S blocks of C are protected GEMMs of their own (every BS x BS block
 // lies in exactly one of them, so the check is unchanged).  Host->device copies run on a copy
-// stream in the order A0, B0, A1, B1, ..., the compute stream starts block (i, j) as soon as
-// A_i and B_j have landed (encode of a slab / panel runs once), and each finished C block is
+// stream in the order A0, B0, B1, A1, ..., B(S-1), A(S-1), the compute stream starts block
+// (i, j) as soon as A_i and B_j have landed (encode of a slab / panel runs once), and each
+// finished C block is
 // copied back on a third stream -- PCIe in both directions overlaps the DMMA GEMMs.
 namespace {
 constexpr int kMaxSplit = 8, kDefaultSplit = 4;
@@ -500,19 +501,32 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
   if (cudaEventRecord(evStart, st) != cudaSuccess || cudaStreamWaitEvent(hp.in, evStart, 0) != cudaSuccess ||
       cudaStreamWaitEvent(hp.out, evStart, 0) != cudaSuccess)
     return check_launch("pipeline start");
-  // host -> device: A0, B0, A1, B1, ...
+  // host -> device in the order A0, B0, B1, A1, B2, A2, ..., B(S-1), A(S-1): every piece after
+  // the first pair unlocks GEMM blocks at once, and the last one (an A slab) unlocks only one
+  // block-row, so the work left after the final copy is S blocks rather than 2S - 1
+  int ord_kind[2 * kMaxSplit], ord_idx[2 * kMaxSplit];  // kind 0 = A slab, 1 = B panel
   for (int i = 0; i < S; ++i) {
-    const int64_t mi = piece(M, sp.ms, i), nj = piece(N, sp.ns, i);
-    if (mi > 0 && cudaMemcpy2DAsync(base + a.oA + (size_t)(i * sp.ms) * a.lda * es, a.lda * es,
-                                    static_cast<const char *>(A_host) + (size_t)(i * sp.ms) * K * es,
-                                    K * es, K * es, mi, cudaMemcpyHostToDevice, hp.in) != cudaSuccess)
-      return check_launch("host->device copy (A)");
-    cudaEventRecord(evA[i], hp.in);
-    if (nj > 0 && cudaMemcpy2DAsync(base + a.oB + (size_t)(i * sp.ns) * es, a.ldb * es,
-                                    static_cast<const char *>(B_host) + (size_t)(i * sp.ns) * es,
-                                    N * es, nj * es, K, cudaMemcpyHostToDevice, hp.in) != cudaSuccess)
-      return check_launch("host->device copy (B)");
-    cudaEventRecord(evB[i], hp.in);
+    ord_kind[2 * i] = i == 0 ? 0 : 1;
+    ord_kind[2 * i + 1] = i == 0 ? 1 : 0;
+    ord_idx[2 * i] = ord_idx[2 * i + 1] = i;
+  }
+  for (int o = 0; o < 2 * S; ++o) {
+    const int i = ord_idx[o];
+    if (ord_kind[o] == 0) {
+      const int64_t mi = piece(M, sp.ms, i);
+      if (mi > 0 && cudaMemcpy2DAsync(base + a.oA + (size_t)(i * sp.ms) * a.lda * es, a.lda * es,
+                                      static_cast<const char *>(A_host) + (size_t)(i * sp.ms) * K * es,
+                                      K * es, K * es, mi, cudaMemcpyHostToDevice, hp.in) != cudaSuccess)
+        return check_launch("host->device copy (A)");
+      cudaEventRecord(evA[i], hp.in);
+    } else {
+      const int64_t nj = piece(N, sp.ns, i);
+      if (nj > 0 && cudaMemcpy2DAsync(base + a.oB + (size_t)(i * sp.ns) * es, a.ldb * es,
+                                      static_cast<const char *>(B_host) + (size_t)(i * sp.ns) * es,
+                                      N * es, nj * es, K, cudaMemcpyHostToDevice, hp.in) != cudaSuccess)
+        return check_launch("host->device copy (B)");
+      cudaEventRecord(evB[i], hp.in);
+    }
   }
   const size_t wsb = aabft_workspace_bytes(cfg);
   auto *cnt_blocks = reinterpret_cast<aabft_counts *>(base + a.oCnt);
@@ -524,12 +538,12 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
   size_t rcol_off = 0, rrow_off = 0, rep_off = 0;
   bool encA[kMaxSplit] = {}, encB[kMaxSplit] = {};
   int nblk = 0;
-  // compute order: diagonal shells, so block (i, j) runs as soon as A_i and B_j are resident
-  for (int d = 0; d < S; ++d) {
-    for (int t = 0; t <= 2 * d; ++t) {
-      const int i = t <= d ? d : t - d - 1, j = t <= d ? t : d;
+  // compute order = arrival order: each piece runs the blocks it completes, so block (i, j)
+  // starts as soon as both A_i and B_j are resident
+  auto run_block = [&](int i, int j) -> aabft_status {
       const int64_t mi = piece(M, sp.ms, i), nj = piece(N, sp.ns, j);
-      if (mi <= 0 || nj <= 0) continue;
+      if (mi <= 0 || nj <= 0) return AABFT_OK;
+      aabft_status s;
       aabft_config cb = *cfg;
       cb.M = mi;
       cb.N = nj;
@@ -568,6 +582,16 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
                             N * es, prod.C, a.ldc * es, nj * es, mi, cudaMemcpyDeviceToHost, hp.out) != cudaSuccess)
         return check_launch("device->host copy (C)");
       ++nblk;
+      return AABFT_OK;
+  };
+  bool haveA[kMaxSplit] = {}, haveB[kMaxSplit] = {};
+  for (int o = 0; o < 2 * S; ++o) {
+    const int x = ord_idx[o];
+    (ord_kind[o] == 0 ? haveA : haveB)[x] = true;
+    for (int y = 0; y < S; ++y) {
+      const bool other = ord_kind[o] == 0 ? haveB[y] : haveA[y];
+      if (!other) continue;
+      if ((s = ord_kind[o] == 0 ? run_block(x, y) : run_block(y, x)) != AABFT_OK) return s;
     }
   }
   // global counters = sum over the blocks (SUM n, MAX max_ratio)
