@@ -8,6 +8,7 @@
 #include <cstdio>
 #include <cstring>
 #include <new>
+#include <vector>
 
 #include "common.cuh"
 
@@ -501,6 +502,20 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
   if (cudaEventRecord(evStart, st) != cudaSuccess || cudaStreamWaitEvent(hp.in, evStart, 0) != cudaSuccess ||
       cudaStreamWaitEvent(hp.out, evStart, 0) != cudaSuccess)
     return check_launch("pipeline start");
+  // AABFT_HOST_TRACE=1: timing events per copy / block, printed to stderr after the call
+  // (diagnostics for the pipeline's schedule; no effect on results)
+  static const bool trace = std::getenv("AABFT_HOST_TRACE") != nullptr;
+  struct Mark { cudaEvent_t e; char what[24]; };
+  std::vector<Mark> marks;
+  auto mark = [&](cudaStream_t on, const char *what, int x, int y) {
+    if (!trace) return;
+    Mark m;
+    cudaEventCreate(&m.e);
+    cudaEventRecord(m.e, on);
+    std::snprintf(m.what, sizeof m.what, "%s %d %d", what, x, y);
+    marks.push_back(m);
+  };
+  mark(st, "start", 0, 0);
   // host -> device in the order A0, B0, B1, A1, B2, A2, ..., B(S-1), A(S-1): every piece after
   // the first pair unlocks GEMM blocks at once, and the last one (an A slab) unlocks only one
   // block-row, so the work left after the final copy is S blocks rather than 2S - 1
@@ -519,6 +534,7 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
                                       K * es, K * es, mi, cudaMemcpyHostToDevice, hp.in) != cudaSuccess)
         return check_launch("host->device copy (A)");
       cudaEventRecord(evA[i], hp.in);
+      mark(hp.in, "h2d A", i, 0);
     } else {
       const int64_t nj = piece(N, sp.ns, i);
       if (nj > 0 && cudaMemcpy2DAsync(base + a.oB + (size_t)(i * sp.ns) * es, a.ldb * es,
@@ -526,6 +542,7 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
                                       N * es, nj * es, K, cudaMemcpyHostToDevice, hp.in) != cudaSuccess)
         return check_launch("host->device copy (B)");
       cudaEventRecord(evB[i], hp.in);
+      mark(hp.in, "h2d B", i, 0);
     }
   }
   const size_t wsb = aabft_workspace_bytes(cfg);
@@ -577,10 +594,12 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
       if ((s = aabft_correct(&cb, &enc, &prod, rep, cnt, stream)) != AABFT_OK) return s;
       // device -> host of the finished (corrected) C block on the copy-out stream
       cudaEventRecord(evC[nblk], st);
+      mark(st, "block done", i, j);
       cudaStreamWaitEvent(hp.out, evC[nblk], 0);
       if (cudaMemcpy2DAsync(static_cast<char *>(C_host) + ((size_t)(i * sp.ms) * N + (size_t)(j * sp.ns)) * es,
                             N * es, prod.C, a.ldc * es, nj * es, mi, cudaMemcpyDeviceToHost, hp.out) != cudaSuccess)
         return check_launch("device->host copy (C)");
+      mark(hp.out, "d2h", i, j);
       ++nblk;
       return AABFT_OK;
   };
@@ -602,6 +621,14 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
   cudaEventRecord(evOutDone, hp.out);
   cudaStreamWaitEvent(st, evOutDone, 0);
   if (cudaStreamSynchronize(st) != cudaSuccess) return check_launch("stream sync");
+  if (trace) {
+    for (auto &m : marks) {
+      float ms = 0.f;
+      cudaEventElapsedTime(&ms, marks[0].e, m.e);
+      std::fprintf(stderr, "[aabft host trace] %8.3f ms  %s\n", ms, m.what);
+    }
+    for (auto &m : marks) cudaEventDestroy(m.e);
+  }
   return AABFT_OK;
   AABFT_GUARD_END
 }
