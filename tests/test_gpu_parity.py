@@ -188,8 +188,69 @@ def test_clean_run_verdicts(P, orc, dtype, recipe, fused):
     assert cnt["blocks"] == (M // bs) * (N // bs) == cnt["clean"]
     assert cnt["checks_rounding"] + cnt["checks_tolerable"] == (M // bs) * N + M * (N // bs)
     assert cnt["max_ratio"] < 0.9
+    # every report field and class counter (clean margins are far from sigma: all ROUNDING)
+    assert_reports_equal(rep, o["check"])
+    assert [cnt["checks_rounding"], cnt["checks_tolerable"], cnt["checks_critical"]] == \
+        o["check"].counts[5:8].tolist()
     if recipe == "integer":
         assert cnt["max_ratio"] == 0.0 and cnt["checks_rounding"] == o["check"].counts[5]
+
+
+def assert_reports_equal(rep, och, mask=None, ratio=False):
+    """Block reports GPU vs oracle, field by field (status, worst class, bad row / column
+    counts, located element; optionally max |d|/eps to float precision)."""
+    m = np.ones(rep.shape, bool) if mask is None else mask
+    for g, o in (("status", "status"), ("worst_class", "worst"), ("n_bad_rows", "nrows"),
+                 ("n_bad_cols", "ncols"), ("row", "row"), ("col", "col")):
+        gv, ov = rep[g][m].astype(np.int64), getattr(och, o)[m].astype(np.int64)
+        assert np.array_equal(gv, ov), (g, np.argwhere(m)[np.flatnonzero(gv != ov)][:5],
+                                        gv[gv != ov][:5], ov[gv != ov][:5])
+    if ratio:
+        gr, orr = rep["max_ratio"][m].astype(np.float64), och.ratio[m]
+        fin = np.isfinite(orr)
+        assert np.array_equal(np.isfinite(gr), fin)
+        assert np.allclose(gr[fin], orr[fin], rtol=2e-6, atol=0), np.max(np.abs(gr[fin] / orr[fin] - 1))
+
+
+@pytest.mark.parametrize("dtype,fused,bs", [(np.float64, True, 8), (np.float64, True, 16),
+                                            (np.float64, True, 32), (np.float64, True, 64),
+                                            (np.float64, False, 64), (np.float64, False, 128),
+                                            (np.float32, False, 8), (np.float32, False, 64)])
+def test_three_classes_every_field(P, orc, dtype, fused, bs):
+    """The runtime classes (reading R10) at block granularity: integer data and a
+    small t make d equal the realised fault error, faults at 0.5 / 2 / 4 sigma of one check
+    per block give ROUNDING, TOLERABLE and CRITICAL checks; every report field, the three
+    class counters and the per-block max |d|/eps must equal the oracle's, and the expected
+    values (paper definitions on realised errors, tests/test_oracle_classes.py) too."""
+    from test_oracle_classes import class_fault_set
+    M, N, K, p = 256, 384, 96, 2
+    t = 20 if dtype == np.float64 else 10
+    A = gen("integer", M, K, 17, 0, dtype, q=5)
+    B = gen("integer", K, N, 17, 1, dtype, q=5)
+    faults, exp, ncls = class_fault_set(orc, A, B, bs, p, t, 3.0, np.random.default_rng(bs))
+    assert ncls[1] > 0 and ncls[2] > 0
+    plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p, t=t, fused=fused)
+    fl = [dict(row=f["row"], col=f["col"], site=2, add=f["add"]) for f in faults]
+    res = plan.run(to_dev(A), to_dev(B), faults=fl, correct=False)
+    torch.cuda.synchronize()
+    rep, cnt = res.reports(), res.counts()
+    o = orc.protected_matmul(A, B, bs=bs, p=p, t=t, faults=fl, do_correct=False)
+    assert_reports_equal(rep, o["check"], ratio=True)
+    for g, k in (("status", "status"), ("worst_class", "worst"), ("n_bad_rows", "nrows"),
+                 ("n_bad_cols", "ncols"), ("row", "row"), ("col", "col")):
+        assert np.array_equal(rep[g].astype(np.int64), exp[k]), g
+    got = [cnt["checks_rounding"], cnt["checks_tolerable"], cnt["checks_critical"]]
+    assert got == o["check"].counts[5:8].tolist() == ncls.tolist()
+    for k, name in enumerate(("blocks", "clean", "corrected", "checksum_only", "uncorrectable")):
+        assert cnt[name] == o["check"].counts[k], name
+    assert cnt["max_ratio"] == pytest.approx(o["check"].max_ratio, rel=2e-6)
+    # correction of the located blocks (CORRECTED count and exact restoration)
+    res = plan.run(to_dev(A), to_dev(B), faults=fl, correct=True)
+    torch.cuda.synchronize()
+    o2 = orc.protected_matmul(A, B, bs=bs, p=p, t=t, faults=fl, do_correct=True)
+    assert np.array_equal(res.reports()["status"].astype(np.int64), o2["check"].status)
+    assert res.counts()["corrected"] == o2["check"].counts[2] == int((exp["status"] == 4).sum())
+    assert np.array_equal(host(res.C), o2["C"])
 
 
 def _fault_set(orc, A, B, bs, p, rng, dtype, n_per_mag=1):
@@ -250,6 +311,7 @@ def test_fault_verdicts_outside_band(P, orc, dtype, fused, bs):
     ost = o["check"].status
     Cg = host(res.C)
     nchk = 0
+    nonband = np.zeros(ost.shape, bool)
     for f, lab in zip(faults, labels):
         I, J = f["row"] // bs, f["col"] // bs
         g, og = rep["status"][I, J], ost[I, J]
@@ -275,7 +337,18 @@ def test_fault_verdicts_outside_band(P, orc, dtype, fused, bs):
         if lab != "band":
             assert g == og, (f, lab, g, og)
             nchk += 1
+            nonband[I, J] = True
     assert nchk > len(faults) // 2
+    # located element and bad row / column counts of every non-band block (their worst class
+    # may sit at the sigma edge for a 'silent' fault, so it is compared where the fault is
+    # critical: then every side is CRITICAL)
+    och = o["check"]
+    for fld, ofld in (("n_bad_rows", "nrows"), ("n_bad_cols", "ncols"), ("row", "row"),
+                      ("col", "col")):
+        assert np.array_equal(rep[fld][nonband].astype(np.int64),
+                              getattr(och, ofld)[nonband].astype(np.int64)), fld
+    crit = nonband & (ost != 0)
+    assert np.array_equal(rep["worst_class"][crit], och.worst[crit])
     # untouched elements are bit-identical to the clean run
     mask = np.ones_like(Cg, bool)
     for f in faults:
