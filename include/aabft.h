@@ -71,8 +71,18 @@ typedef struct {
   int32_t t;
   double omega;
   int32_t fma_model;
-  int32_t reserved;
+  int32_t flags;  /* AABFT_FLAG_* (0 = defaults) */
 } aabft_config;
+
+/* AABFT_FLAG_TOPP_IN_GEMM: move the top-p selection of step 1 (Alg 1) from
+ * aabft_encode into aabft_gemm, which takes it from the operand tiles it already streams
+ * through shared memory -- the paper runs this reduction "in parallel to the matrix
+ * multiplication kernel".  Honoured where the GEMM supports it (FP64,
+ * p <= 4); elsewhere aabft_encode selects as usual.  Either way the top-p tables of
+ * aabft_encoded are complete once aabft_gemm (stream-ordered) has run, with identical
+ * contents (value desc, index asc; bit-exact).  Opt-in: on B200 it measured slower than the
+ * selection in aabft_encode. */
+#define AABFT_FLAG_TOPP_IN_GEMM 1
 
 /* Output of aabft_encode.  Acs: (M/bs) x K, ld_acs >= K.  Bcs: K x (N/bs), ld_bcs >= N/bs.
  * topA_val/topA_idx: (M + M/bs) x p -- data rows 0..M-1, then checksum rows; |value|

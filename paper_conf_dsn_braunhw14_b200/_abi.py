@@ -17,6 +17,7 @@ LIB_PATH = os.environ.get("AABFT_LIB", os.path.join(HERE, "libaabft.so"))
 F64, F32 = 0, 1
 BLK_CLEAN, BLK_CORRECTED, BLK_CHECKSUM_ONLY, BLK_UNCORRECTABLE, BLK_SINGLE = 0, 1, 2, 3, 4
 STATUS_NAMES = {0: "CLEAN", 1: "CORRECTED", 2: "CHECKSUM_ONLY", 3: "UNCORRECTABLE", 4: "SINGLE"}
+FLAG_TOPP_IN_GEMM = 1  # include/aabft.h AABFT_FLAG_TOPP_IN_GEMM
 COUNT_NAMES = ("blocks", "clean", "corrected", "checksum_only", "uncorrectable",
                "checks_rounding", "checks_tolerable", "checks_critical")
 EXPORTED = ("aabft_workspace_bytes", "aabft_encode", "aabft_bound", "aabft_bound_elements",
@@ -30,7 +31,7 @@ EXPORTED = ("aabft_workspace_bytes", "aabft_encode", "aabft_bound", "aabft_bound
 class Config(C.Structure):
     _fields_ = [("dtype", C.c_int32), ("bs", C.c_int32), ("M", C.c_int64), ("N", C.c_int64),
                 ("K", C.c_int64), ("p", C.c_int32), ("t", C.c_int32), ("omega", C.c_double),
-                ("fma_model", C.c_int32), ("reserved", C.c_int32)]
+                ("fma_model", C.c_int32), ("flags", C.c_int32)]
 
 
 class Encoded(C.Structure):

@@ -113,12 +113,18 @@ class ProtectedGemm:
 
     def __init__(self, M: int, N: int, K: int, *, dtype=torch.float64, bs: int = 64, p: int = 2,
                  omega: float = 3.0, t: int = 0, fma_model: int = 1, device=None,
-                 fused: bool = True):
+                 fused: bool = True, topp_in_gemm: bool = False):
         lib()  # fail loudly before allocating anything
         self.device = torch.device("cuda" if device is None else device)
         self.dtype = dtype
         self.M, self.N, self.K, self.bs, self.p = M, N, K, bs, p
         self.cfg = Config(_dtype_code(dtype), bs, M, N, K, p, t, omega, fma_model, 0)
+        # AABFT_FLAG_TOPP_IN_GEMM (include/aabft.h): run() lets the GEMM select the top-p
+        # (opt-in: measured slower than selecting in the encode pass)
+        self.topp_in_gemm = bool(topp_in_gemm)
+        self.cfg_defer = Config(_dtype_code(dtype), bs, M, N, K, p, t, omega, fma_model,
+                                _abi.FLAG_TOPP_IN_GEMM)
+        self._topp_pending = False
         dev, dt = self.device, dtype
         nI, nJ = M // bs, N // bs
         self.ld_acs = _pad_ld(K, dt)
@@ -184,17 +190,23 @@ class ProtectedGemm:
             raise ValueError(f"{name} must be row-major (stride(1) == 1)")
 
     # --- the four steps (each one C-ABI call)
-    def encode(self, A, B, stream=None, topp: bool = True):
-        """Step 1; topp=False encodes the checksums only (fixed-eps / SEA comparators)."""
+    def encode(self, A, B, stream=None, topp: bool = True, defer: bool = False):
+        """Step 1; topp=False encodes the checksums only (fixed-eps / SEA comparators);
+        defer=True leaves the top-p selection to the following gemm() where the library
+        supports it (AABFT_FLAG_TOPP_IN_GEMM; the tables are complete after gemm())."""
         L = lib()
         s = _stream_ptr(stream)
-        ok(L.aabft_encode(C.byref(self.cfg), _ptr(A), A.stride(0) if A is not None else 0,
+        self._topp_pending = bool(defer and topp)
+        cfg = self.cfg_defer if self._topp_pending else self.cfg
+        ok(L.aabft_encode(C.byref(cfg), _ptr(A), A.stride(0) if A is not None else 0,
                           _ptr(B), B.stride(0) if B is not None else 0,
                           C.byref(self.enc if topp else self.enc_cs),
                           self.ws.data_ptr(), self.ws_bytes, s), "aabft_encode")
 
     def gemm(self, A, B, faults: torch.Tensor | None = None, nfaults: int = 0, stream=None):
-        ok(lib().aabft_gemm(C.byref(self.cfg), A.data_ptr(), A.stride(0), B.data_ptr(),
+        cfg = self.cfg_defer if self._topp_pending else self.cfg
+        self._topp_pending = False
+        ok(lib().aabft_gemm(C.byref(cfg), A.data_ptr(), A.stride(0), B.data_ptr(),
                             B.stride(0), C.byref(self.enc), C.byref(self.prod), _ptr(faults),
                             nfaults, self.ws.data_ptr(), self.ws_bytes, _stream_ptr(stream)),
            "aabft_gemm")
@@ -303,7 +315,7 @@ class ProtectedGemm:
         self._check_operand(B, self.K, self.N, "B")
         fbuf = faults if isinstance(faults, torch.Tensor) else make_faults(faults, self.device)
         nf = 0 if fbuf is None else fbuf.numel() // 48
-        self.encode(A, B, stream)
+        self.encode(A, B, stream, defer=self.topp_in_gemm)
         self.gemm(A, B, fbuf, nf, stream)
         self.check(stream)
         if correct:

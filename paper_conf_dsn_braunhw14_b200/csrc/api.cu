@@ -82,6 +82,8 @@ aabft_status validate(const aabft_config *c) {
   if (c->t < 0 || c->t > 200) { set_error("t=%d out of range", c->t); return AABFT_EINVAL; }
   if (c->fma_model != 0 && c->fma_model != 1) { set_error("fma_model must be 0 or 1"); return AABFT_EINVAL; }
   if ((c->M / c->bs) * (c->N / c->bs) >= ((int64_t)1 << 31)) { set_error("too many blocks"); return AABFT_EINVAL; }
+  // launch-geometry limit (gridDim.y <= 65535): block-rows of A in the streaming check
+  if (c->M / c->bs > 65535) { set_error("M/bs = %lld exceeds 65535 block-rows", (long long)(c->M / c->bs)); return AABFT_EINVAL; }
   return AABFT_OK;
 }
 

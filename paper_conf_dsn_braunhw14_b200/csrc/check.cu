@@ -521,6 +521,15 @@ __global__ void correct_kernel(CheckArgs a, BoundParams bp, T *C) {
     for (int64_t jj = J * bs; jj < J * bs + bs; ++jj) ref = ref + (double)C[i * a.ldc + jj];
     const double d = ref - (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
     const Bound b = row_bound<EXT, P>(a, bp, i, J);
+    if (a.Rcol) {
+      // fused check: the epilogue reference sums still describe the faulty element; refresh
+      // the two that pass through (i, j) from the corrected C so a later aabft_check of the
+      // same product sees the corrected state (ascending order, double)
+      double rc = 0.0;
+      for (int64_t ii = I * bs; ii < I * bs + bs; ++ii) rc = rc + (double)C[ii * a.ldc + j];
+      const_cast<double *>(a.Rcol)[I * a.N + j] = rc;
+      const_cast<double *>(a.Rrow)[i * nJ + J] = ref;
+    }
     unsigned long long *n = reinterpret_cast<unsigned long long *>(a.cnt->n);
     if (fabs(d) <= b.eps) {
       r->status = AABFT_BLK_CORRECTED;
@@ -558,6 +567,14 @@ CheckArgs make_args(const aabft_config *cfg, const aabft_encoded *enc, const aab
     a.Rrow2 = rr2;
   }
   return a;
+}
+
+// correction: the fused reference sums (complete after aabft_check) are refreshed for every
+// corrected element (a second check of a corrected product must stay clean)
+void set_refresh(const aabft_config *cfg, const aabft_product *prod, CheckArgs &a) {
+  const bool fused = prod->Rcol && prod->Rrow && cfg->dtype == AABFT_F64 && cfg->bs <= 64;
+  a.Rcol = fused ? prod->Rcol : nullptr;
+  a.Rrow = fused ? prod->Rrow : nullptr;
 }
 
 template <typename T, int P, bool EXT = false>
@@ -683,7 +700,8 @@ aabft_status launch_correct(const aabft_config *cfg, const aabft_encoded *enc,
                             const aabft_product *prod, aabft_block_report *rep,
                             aabft_counts *cnt, cudaStream_t st) {
   const BoundParams bp = make_bound_params(cfg);
-  const CheckArgs a = make_args(cfg, enc, prod, rep, cnt);
+  CheckArgs a = make_args(cfg, enc, prod, rep, cnt);
+  set_refresh(cfg, prod, a);
   if (cfg->dtype == AABFT_F64) {
     AABFT_P_SWITCH(cfg->p, return (run_correct<double, PP>(cfg, a, bp, st)));
   } else {
@@ -715,6 +733,7 @@ aabft_status launch_correct_ext(const aabft_config *cfg, const aabft_product *pr
                                 aabft_counts *cnt, cudaStream_t st) {
   const BoundParams bp = make_bound_params(cfg);
   CheckArgs a = make_args(cfg, nullptr, prod, rep, cnt);
+  set_refresh(cfg, prod, a);
   a.eps_row = eps_row;
   a.eps_fixed = eps_fixed;
   if (cfg->dtype == AABFT_F64) return run_correct<double, 1, true>(cfg, a, bp, st);

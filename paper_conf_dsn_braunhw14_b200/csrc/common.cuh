@@ -53,6 +53,7 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
 size_t encode_ws_bytes(const aabft_config *cfg);
 aabft_status launch_counts_sum(const aabft_counts *parts, int n, aabft_counts *out, cudaStream_t st);
 size_t gemm_f64_ws_bytes(const aabft_config *cfg);
+bool gemm_f64_topp_ok(const aabft_config *cfg);  // AABFT_FLAG_TOPP_IN_GEMM honoured
 void gemm_f64_red_ptrs(const aabft_config *cfg, void *gemm_ws, double **rcol2, double **rrow2);
 int gemm_f64_fused_parts(int bs, int *row_parts);  // returns column parts
 aabft_status launch_gemm_f32(const aabft_config *cfg, const void *A, int64_t lda,
@@ -132,6 +133,29 @@ __device__ __forceinline__ void tp_push(double (&v)[P], int (&ix)[P], double a, 
   } else {
     if (a > v[P - 1]) tp_insert<P>(v, ix, a, idx);
   }
+}
+
+// tp_push on the bit patterns of |x|: for non-negative doubles the unsigned 64-bit order of
+// the bits is the value order, so the selection runs on the integer ALU (ISETP/SEL) instead
+// of the FP64 pipe -- which the FP64 GEMM keeps busy with DMMA.  Same list as tp_push.
+template <int P>
+__device__ __forceinline__ void tp_push_bits(unsigned long long (&v)[P], int (&ix)[P],
+                                             unsigned long long a, int idx) {
+  bool g[P];
+#pragma unroll
+  for (int r = 0; r < P; ++r) g[r] = a > v[r];
+#pragma unroll
+  for (int r = P - 1; r >= 1; --r) {
+    const unsigned long long vr = g[r - 1] ? v[r - 1] : (g[r] ? a : v[r]);
+    const int ir = g[r - 1] ? ix[r - 1] : (g[r] ? idx : ix[r]);
+    v[r] = vr;
+    ix[r] = ir;
+  }
+  v[0] = g[0] ? a : v[0];
+  ix[0] = g[0] ? idx : ix[0];
+}
+__device__ __forceinline__ unsigned long long abs_bits(double x) {
+  return (unsigned long long)__double_as_longlong(x) & 0x7FFFFFFFFFFFFFFFull;
 }
 
 template <int P>

@@ -5,15 +5,21 @@
 // B200 design: HBM-bound streaming.  One thread owns one column of a
 // BS-row block of A, so the column checksum is a register running sum in ascending row order
 // (bit-identical to Eq 1 summed top -> bottom, reading R11) and every warp load is a
-// contiguous 256 B row segment.  The same pass stages |a| in padded shared memory where four
-// lanes per row keep register top-p lists over interleaved columns and merge them with two
-// xor-shuffles (warp-shuffle top-p).  B is the mirror image: a thread owns a column of B
-// (running top-p over k in registers) and the BS-wide row sums are taken from the staged
-// tile, one sequential thread per (row, block).  Partial top-p lists per chunk are reduced
-// by a warp-per-vector kernel that also computes the top-p of the checksum vectors.
-// Strips are double-buffered in registers (the next strip's loads are in flight during the
-// top-p / row-sum phase) and the top-p insertion is branch-free for p <= 4 (tp_push), so a
-// warp never diverges on inserts: 44 + 43 + 9 us at 4096^2 FP64.
+// contiguous 256 B row segment.  The same pass stages the selection KEYS of |a| in padded
+// shared memory, where four lanes per row keep register top-p lists over interleaved columns
+// and merge them with two xor-shuffles (warp-shuffle top-p).  B is the mirror image: a thread
+// owns a column of B (running top-p over k in registers) and the BS-wide row sums are taken
+// from the staged tile, one sequential thread per (row, block).
+//  * Selection keys: the bit pattern of |x| (+1) as an unsigned integer orders like |x|, so
+//    the top-p compares and selects run on the integer ALU (ISETP/SEL) rather than the FP64
+//    pipe (FP32 data: 32-bit keys); the insertion is branch-free (kp_push), so a warp never
+//    diverges on inserts.
+//  * Each CTA parks its chunk's partial lists; step 3 merges them with a warp per vector
+//    across the whole GPU (topp_reduce_kernel).  A last-CTA-per-group merge inside the encode
+//    launches was measured slower: the merges serialise on L2 latency in a few CTAs
+//    (DESIGN.md 8.7).
+//  * Strips are double-buffered in registers (the next strip's loads are in flight during the
+//    top-p / row-sum phase).
 #include <algorithm>
 
 #include "common.cuh"
@@ -21,35 +27,136 @@
 namespace aabft {
 namespace {
 
-constexpr int kStrip = 32;  // rows staged per pass
+#ifndef AABFT_ENC_STRIP
+#define AABFT_ENC_STRIP 32
+#endif
+constexpr int kStrip = AABFT_ENC_STRIP;  // rows staged per pass
 
 template <typename T>
 __device__ __forceinline__ T ldg(const T *p) { return __ldg(p); }
 
+// ------------------------------------------------------------------------- selection keys
+template <typename T> struct Key;
+template <> struct Key<double> {
+  using type = unsigned long long;
+  static __device__ __forceinline__ type of(double x) {
+    return ((unsigned long long)__double_as_longlong(x) & 0x7FFFFFFFFFFFFFFFull) + 1ull;
+  }
+  static __device__ __forceinline__ double val(type k) { return __longlong_as_double((long long)(k - 1ull)); }
+};
+template <> struct Key<float> {
+  using type = unsigned int;
+  static __device__ __forceinline__ type of(float x) { return (__float_as_uint(x) & 0x7FFFFFFFu) + 1u; }
+  static __device__ __forceinline__ double val(type k) { return (double)__uint_as_float(k - 1u); }
+};
+
+// key 0 with index -1 is below every element (keys are >= 1)
+template <int P, typename KT>
+__device__ __forceinline__ void kp_init(KT (&v)[P], int (&ix)[P]) {
+#pragma unroll
+  for (int r = 0; r < P; ++r) { v[r] = 0; ix[r] = -1; }
+}
+
+// push an element that loses every tie (larger index than everything in the list: a lane
+// scanning its own elements in ascending index order); branch-free for every P
+template <int P, typename KT>
+__device__ __forceinline__ void kp_push(KT (&v)[P], int (&ix)[P], KT a, int idx) {
+  bool g[P];
+#pragma unroll
+  for (int r = 0; r < P; ++r) g[r] = a > v[r];
+#pragma unroll
+  for (int r = P - 1; r >= 1; --r) {
+    const KT vr = g[r - 1] ? v[r - 1] : (g[r] ? a : v[r]);
+    const int ir = g[r - 1] ? ix[r - 1] : (g[r] ? idx : ix[r]);
+    v[r] = vr;
+    ix[r] = ir;
+  }
+  v[0] = g[0] ? a : v[0];
+  ix[0] = g[0] ? idx : ix[0];
+}
+
+// insertion with the full order (key desc, index asc; empty slots have index -1 and key 0)
+template <int P, typename KT>
+__device__ __forceinline__ void kp_insert(KT (&v)[P], int (&ix)[P], KT a, int idx) {
+  if (idx < 0) return;
+#pragma unroll
+  for (int r = 0; r < P; ++r) {
+    const bool better = a > v[r] || (a == v[r] && (ix[r] < 0 || idx < ix[r]));
+    if (better) {
+      const KT tv = v[r];
+      const int ti = ix[r];
+      v[r] = a;
+      ix[r] = idx;
+      a = tv;
+      idx = ti;
+      if (idx < 0) break;
+    }
+  }
+}
+
+template <int P, typename KT>
+__device__ __forceinline__ void kp_shfl_merge(KT (&v)[P], int (&ix)[P], int lane_mask) {
+  KT ov[P];
+  int oi[P];
+#pragma unroll
+  for (int r = 0; r < P; ++r) {
+    ov[r] = __shfl_xor_sync(0xffffffffu, v[r], lane_mask);
+    oi[r] = __shfl_xor_sync(0xffffffffu, ix[r], lane_mask);
+  }
+#pragma unroll
+  for (int r = 0; r < P; ++r) kp_insert<P, KT>(v, ix, ov[r], oi[r]);
+}
+
+template <typename T, int P>
+__device__ __forceinline__ void kp_store(double *dv, int *di, const typename Key<T>::type (&v)[P],
+                                         const int (&ix)[P]) {
+#pragma unroll
+  for (int s = 0; s < P; ++s) {
+    dv[s] = ix[s] < 0 ? -1.0 : Key<T>::val(v[s]);
+    di[s] = ix[s];
+  }
+}
+
+// Step 3 for one vector: merge its `nch` partial lists (value desc, index asc) with a warp and
+// write the final p entries.  Partial lists come from other CTAs: read them through L2.
+template <int P>
+__device__ __forceinline__ void merge_vector(const double *__restrict__ pv, const int *__restrict__ pi,
+                                             int nch, double *ov, int *oi, int lane) {
+  double v[P];
+  int ix[P];
+  tp_init<P>(v, ix);
+  for (int e = lane; e < nch * P; e += 32) tp_insert<P>(v, ix, __ldcg(pv + e), __ldcg(pi + e));
+#pragma unroll
+  for (int m = 16; m >= 1; m >>= 1) tp_shfl_merge<P>(v, ix, m);
+  if (lane == 0) {
+#pragma unroll
+    for (int s = 0; s < P; ++s) { ov[s] = v[s]; oi[s] = ix[s]; }
+  }
+}
+
 // ---------------------------------------------------------------------------------- A
-// grid (chunks of 128 columns, M/bs block-rows); 128 threads.
+// 1-D grid: unit u -> block-row I = u / nch, column chunk = u % nch (128 columns); 128 threads.
 template <typename T, int P, bool TOPP>
 __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, int64_t lda,
-                                                       int64_t K, int bs, T *__restrict__ Acs,
-                                                       int64_t ld_acs, double *__restrict__ pv,
+                                                       int64_t M, int64_t K, int bs,
+                                                       T *__restrict__ Acs, int64_t ld_acs,
+                                                       double *__restrict__ pv,
                                                        int *__restrict__ pi, int nch) {
-  __shared__ double tile[kStrip][kEncAChunk + 4];  // |A| strip; stride 132 -> conflict-free
+  using KT = typename Key<T>::type;
+  __shared__ KT tile[kStrip][kEncAChunk + 4];  // keys of |A| strip; conflict-free lane reads
   const int c = threadIdx.x;
-  const int chunk = blockIdx.x;
-  const int64_t I = blockIdx.y;
+  const int chunk = (int)(blockIdx.x % (unsigned)nch);
+  const int64_t I = blockIdx.x / (unsigned)nch;
   const int64_t k = (int64_t)chunk * kEncAChunk + c;
   const bool kin = k < K;
   const int r = c >> 2, q = c & 3;  // top-p role: row r of the strip, column phase q
   T sum = T(0);
-  // register double buffering: the loads of strip r0 + kStrip are issued right after strip r0
-  // has been summed and staged, so they are in flight during its top-p phase
   T vals[kStrip];
   auto load_strip = [&](int r0) {
     const int rows = min(kStrip, bs - r0);
     const T *src = A + (I * bs + r0) * lda + k;
     if (rows == kStrip) {
-      // full strip: the kStrip loads are issued back to back (memory-level parallelism; a
-      // per-row guard made the checksums-only instantiation compile to load -> add chains)
+      // full strip: the kStrip loads are issued back to back (memory-level parallelism)
 #pragma unroll
       for (int rr = 0; rr < kStrip; ++rr) vals[rr] = kin ? ldg(src + rr * lda) : T(0);
     } else {
@@ -64,50 +171,46 @@ __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, 
     for (int rr = 0; rr < kStrip; ++rr) {
       if (rr < rows) {
         sum = sum + vals[rr];  // Eq 1, ascending i (Alg 1 line "sum <- sum + Asub[i][tid]")
-        if (TOPP) tile[rr][c] = fabs((double)vals[rr]);
+        if (TOPP) tile[rr][c] = Key<T>::of(vals[rr]);
       }
     }
     if (r0 + kStrip < bs) load_strip(r0 + kStrip);
     if (!TOPP) continue;  // checksums only (fixed-eps / SEA ABFT comparators, NEXT-3)
     __syncthreads();
-    double v[P];
+    KT v[P];
     int ix[P];
-    tp_init<P>(v, ix);
+    kp_init<P>(v, ix);
     if (r < rows) {
-      // ascending columns into this lane's own list: the new element loses every tie.  The
-      // column limit is hoisted (32-bit: K < 2^31 is validated) so the scan carries no
-      // per-element guard or 64-bit index arithmetic.
+      // ascending columns into this lane's own list: the new element loses every tie
       const int kbase = chunk * kEncAChunk;
       const int lim = K - kbase < kEncAChunk ? (int)(K - kbase) : kEncAChunk;
-      const double *trow = tile[r];
-      // (measured: a fully or 8x unrolled version of this loop returned a list holding one
-      // element twice on sm_100a; 4x with the compile-time bound is parity-clean)
-#pragma unroll 4
-      for (int cc = q; cc < kEncAChunk; cc += 4)
-        if (cc < lim) tp_push<P>(v, ix, trow[cc], kbase + cc);
+      const KT *trow = tile[r];
+#pragma unroll 8
+      for (int cc = q; cc < kEncAChunk; cc += 4) {
+        const KT key = cc < lim ? trow[cc] : KT(0);  // key 0 never enters the list
+        kp_push<P, KT>(v, ix, key, kbase + cc);
+      }
     }
-    tp_shfl_merge<P>(v, ix, 1);
-    tp_shfl_merge<P>(v, ix, 2);
+    kp_shfl_merge<P, KT>(v, ix, 1);
+    kp_shfl_merge<P, KT>(v, ix, 2);
     if (r < rows && q == 0) {
       const int64_t row = I * bs + r0 + r;
-      double *dv = pv + (row * nch + chunk) * P;
-      int *di = pi + (row * nch + chunk) * P;
-#pragma unroll
-      for (int s = 0; s < P; ++s) { dv[s] = v[s]; di[s] = ix[s]; }
+      kp_store<T, P>(pv + (row * nch + chunk) * P, pi + (row * nch + chunk) * P, v, ix);
     }
     __syncthreads();
   }
   if (kin) Acs[I * ld_acs + k] = sum;
+  if (!TOPP) return;
   // partial top-p of the checksum row I over this chunk (Alg 1 localSums / maxReduce)
-  if (TOPP) {
-    __shared__ double s_v[kEncAChunk / 32][P];
+  {
+    __shared__ KT s_v[kEncAChunk / 32][P];
     __shared__ int s_i[kEncAChunk / 32][P];
-    double v[P];
+    KT v[P];
     int ix[P];
-    tp_init<P>(v, ix);
-    if (kin) tp_insert<P>(v, ix, fabs((double)sum), (int)k);
+    kp_init<P>(v, ix);
+    if (kin) kp_push<P, KT>(v, ix, Key<T>::of(sum), (int)k);
 #pragma unroll
-    for (int m = 16; m >= 1; m >>= 1) tp_shfl_merge<P>(v, ix, m);
+    for (int m = 16; m >= 1; m >>= 1) kp_shfl_merge<P, KT>(v, ix, m);
     if ((c & 31) == 0) {
 #pragma unroll
       for (int s = 0; s < P; ++s) { s_v[c >> 5][s] = v[s]; s_i[c >> 5][s] = ix[s]; }
@@ -116,39 +219,39 @@ __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, 
     if (c == 0) {
       for (int w = 1; w < kEncAChunk / 32; ++w)
 #pragma unroll
-        for (int s = 0; s < P; ++s) tp_insert<P>(v, ix, s_v[w][s], s_i[w][s]);
-      const int64_t row = (int64_t)gridDim.y * bs + I;  // checksum rows follow the M data rows
-      double *dv = pv + (row * nch + chunk) * P;
-      int *di = pi + (row * nch + chunk) * P;
-#pragma unroll
-      for (int s = 0; s < P; ++s) { dv[s] = v[s]; di[s] = ix[s]; }
+        for (int s = 0; s < P; ++s) kp_insert<P, KT>(v, ix, s_v[w][s], s_i[w][s]);
+      const int64_t row = M + I;  // checksum rows follow the M data rows
+      kp_store<T, P>(pv + (row * nch + chunk) * P, pi + (row * nch + chunk) * P, v, ix);
     }
   }
 }
 
 // ---------------------------------------------------------------------------------- B
-// grid (column chunks of NC, row chunks of kEncBChunk); NC threads (NC = max(128, bs)).
+// 1-D grid: unit u -> column chunk jc = u / nch (NC columns), row chunk kc = u % nch
+// (kEncBChunk rows of B); NC threads (NC = max(128, bs)).
 template <typename T, int P, int NC, bool TOPP>
 __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, int64_t ldb,
                                                       int64_t K, int64_t N, int bs,
                                                       T *__restrict__ Bcs, int64_t ld_bcs,
                                                       double *__restrict__ pv,
                                                       int *__restrict__ pi, int nch) {
+  using KT = typename Key<T>::type;
   constexpr int SB = (NC * sizeof(T) > 1024) ? 16 : kStrip;  // strip rows (smem <= 48 KiB)
   __shared__ T tile[SB][NC + 1];  // odd stride -> conflict-free per-row sequential reads
   const int c = threadIdx.x;
-  const int64_t j = (int64_t)blockIdx.x * NC + c;
+  const int64_t jc = blockIdx.x / (unsigned)nch;
+  const int kc = (int)(blockIdx.x % (unsigned)nch);
+  const int64_t j = jc * NC + c;
   const bool jin = j < N;
-  const int kc = blockIdx.y;
   const int64_t kbeg = (int64_t)kc * kEncBChunk;
   const int64_t kend = K < kbeg + kEncBChunk ? K : kbeg + kEncBChunk;
   const int nblk = NC / bs;  // checksum blocks covered by this CTA (<= 16)
-  __shared__ double s_cv[16][P];
+  __shared__ KT s_cv[16][P];
   __shared__ int s_ci[16][P];
-  if (c < 16 * P) { s_cv[c / P][c % P] = -1.0; s_ci[c / P][c % P] = -1; }
-  double v[P];
+  if (c < 16 * P) { s_cv[c / P][c % P] = 0; s_ci[c / P][c % P] = -1; }
+  KT v[P];
   int ix[P];
-  tp_init<P>(v, ix);
+  kp_init<P>(v, ix);
   // register double buffering as in encode A: strip k0 + SB is loaded during the row sums
   T vals[SB];
   auto load_strip = [&](int64_t k0) {
@@ -171,14 +274,14 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
       for (int rr = 0; rr < SB; ++rr) {
         tile[rr][c] = vals[rr];
         // ascending k, own list: the new element loses every tie
-        if (TOPP && jin) tp_push<P>(v, ix, fabs((double)vals[rr]), k0i + rr);
+        if (TOPP) kp_push<P, KT>(v, ix, Key<T>::of(vals[rr]), k0i + rr);
       }
     } else {
 #pragma unroll
       for (int rr = 0; rr < SB; ++rr) {
         if (rr < rows) {
           tile[rr][c] = vals[rr];
-          if (TOPP && jin) tp_push<P>(v, ix, fabs((double)vals[rr]), k0i + rr);
+          if (TOPP) kp_push<P, KT>(v, ix, Key<T>::of(vals[rr]), k0i + rr);
         }
       }
     }
@@ -189,22 +292,22 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
     // checksum column J (partial over this k-chunk)
     for (int jb = c >> 5; jb < nblk; jb += NC / 32) {
       const int rr = c & 31;
-      const int64_t J = (int64_t)blockIdx.x * nblk + jb;
-      double lv[P];
+      const int64_t J = jc * nblk + jb;
+      KT lv[P];
       int li[P];
-      tp_init<P>(lv, li);
+      kp_init<P>(lv, li);
       if (rr < rows && J * bs < N) {
         T sm = T(0);
         for (int jj = 0; jj < bs; ++jj) sm = sm + tile[rr][jb * bs + jj];
         Bcs[(k0 + rr) * ld_bcs + J] = sm;
-        if (TOPP) tp_push<P>(lv, li, fabs((double)sm), (int)(k0 + rr));
+        if (TOPP) kp_push<P, KT>(lv, li, Key<T>::of(sm), (int)(k0 + rr));
       }
       if (!TOPP) continue;
 #pragma unroll
-      for (int m = 16; m >= 1; m >>= 1) tp_shfl_merge<P>(lv, li, m);
+      for (int m = 16; m >= 1; m >>= 1) kp_shfl_merge<P, KT>(lv, li, m);
       if (rr == 0) {
 #pragma unroll
-        for (int r = 0; r < P; ++r) tp_insert<P>(lv, li, s_cv[jb][r], s_ci[jb][r]);
+        for (int r = 0; r < P; ++r) kp_insert<P, KT>(lv, li, s_cv[jb][r], s_ci[jb][r]);
 #pragma unroll
         for (int r = 0; r < P; ++r) { s_cv[jb][r] = lv[r]; s_ci[jb][r] = li[r]; }
       }
@@ -212,62 +315,58 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
     __syncthreads();
   }
   if (!TOPP) return;
-  if (c < nblk && ((int64_t)blockIdx.x * nblk + c) * bs < N) {
-    const int64_t J = (int64_t)blockIdx.x * nblk + c;
-    double *dv = pv + ((N + J) * nch + kc) * P;
-    int *di = pi + ((N + J) * nch + kc) * P;
+  if (c < nblk && (jc * nblk + c) * bs < N) {
+    const int64_t J = jc * nblk + c;
+    KT cv[P];
+    int ci[P];
 #pragma unroll
-    for (int r = 0; r < P; ++r) { dv[r] = s_cv[c][r]; di[r] = s_ci[c][r]; }
+    for (int r = 0; r < P; ++r) { cv[r] = s_cv[c][r]; ci[r] = s_ci[c][r]; }
+    kp_store<T, P>(pv + ((N + J) * nch + kc) * P, pi + ((N + J) * nch + kc) * P, cv, ci);
   }
-  if (jin) {
-    double *dv = pv + (j * nch + kc) * P;
-    int *di = pi + (j * nch + kc) * P;
-#pragma unroll
-    for (int s = 0; s < P; ++s) { dv[s] = v[s]; di[s] = ix[s]; }
-  }
+  if (jin) kp_store<T, P>(pv + (j * nch + kc) * P, pi + (j * nch + kc) * P, v, ix);
 }
 
 // ---------------------------------------------------------------------------------- step 3
 // One warp per vector (data rows + checksum rows of A, data cols + checksum cols of B): merge
-// the per-chunk partial lists produced by the encode kernels.
-template <typename T, int P>
+// the per-chunk partial lists produced by the encode kernels (P:L368).
+template <int P>
 __global__ void __launch_bounds__(256) topp_reduce_kernel(
-    int64_t M, int64_t N, int64_t K, int bs, const double *__restrict__ pva,
-    const int *__restrict__ pia, int ncha, const double *__restrict__ pvb,
-    const int *__restrict__ pib, int nchb, const T *__restrict__ Acs, int64_t ld_acs,
-    const T *__restrict__ Bcs, int64_t ld_bcs, double *__restrict__ topA_v,
-    int *__restrict__ topA_i, double *__restrict__ topB_v, int *__restrict__ topB_i, int do_a,
-    int do_b) {
+    int64_t M, int64_t N, int bs, const double *__restrict__ pva, const int *__restrict__ pia,
+    int ncha, const double *__restrict__ pvb, const int *__restrict__ pib, int nchb,
+    double *__restrict__ topA_v, int *__restrict__ topA_i, double *__restrict__ topB_v,
+    int *__restrict__ topB_i, int do_a, int do_b) {
   const int lane = threadIdx.x & 31;
   const int64_t w = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
   const int64_t nA = do_a ? M + M / bs : 0;
   const int64_t nB = do_b ? N + N / bs : 0;
   if (w >= nA + nB) return;
-  double v[P];
-  int ix[P];
-  tp_init<P>(v, ix);
-  double *ov;
-  int *oi;
   if (w < nA) {
-    const double *sv = pva + w * ncha * P;
-    const int *si = pia + w * ncha * P;
-    for (int e = lane; e < ncha * P; e += 32) tp_insert<P>(v, ix, sv[e], si[e]);
-    ov = topA_v + w * P;
-    oi = topA_i + w * P;
+    merge_vector<P>(pva + w * ncha * P, pia + w * ncha * P, ncha, topA_v + w * P, topA_i + w * P, lane);
   } else {
     const int64_t u = w - nA;
-    const double *sv = pvb + u * nchb * P;
-    const int *si = pib + u * nchb * P;
-    for (int e = lane; e < nchb * P; e += 32) tp_insert<P>(v, ix, sv[e], si[e]);
-    ov = topB_v + u * P;
-    oi = topB_i + u * P;
+    merge_vector<P>(pvb + u * nchb * P, pib + u * nchb * P, nchb, topB_v + u * P, topB_i + u * P, lane);
   }
-#pragma unroll
-  for (int m = 16; m >= 1; m >>= 1) tp_shfl_merge<P>(v, ix, m);
-  if (lane == 0) {
-#pragma unroll
-    for (int s = 0; s < P; ++s) { ov[s] = v[s]; oi[s] = ix[s]; }
-  }
+}
+
+// workspace: [A partial values][A partial indices][B values][B indices]
+struct EncWs {
+  double *pva, *pvb;
+  int *pia, *pib;
+};
+
+size_t r256e(size_t b) { return (b + 255) / 256 * 256; }
+
+EncWs enc_ws(const aabft_config *cfg, void *ws) {
+  const size_t p = (size_t)cfg->p;
+  const size_t ncha = (size_t)enc_a_chunks(cfg->K), nchb = (size_t)enc_b_chunks(cfg->K);
+  const size_t ra = (size_t)(cfg->M + cfg->M / cfg->bs), rb = (size_t)(cfg->N + cfg->N / cfg->bs);
+  char *w = static_cast<char *>(ws);
+  EncWs e;
+  e.pva = reinterpret_cast<double *>(w); w += r256e(ra * ncha * p * 8);
+  e.pia = reinterpret_cast<int *>(w); w += r256e(ra * ncha * p * 4);
+  e.pvb = reinterpret_cast<double *>(w); w += r256e(rb * nchb * p * 8);
+  e.pib = reinterpret_cast<int *>(w);
+  return e;
 }
 
 template <typename T, int P>
@@ -276,44 +375,37 @@ aabft_status run_encode(const aabft_config *cfg, const T *A, int64_t lda, const 
   const int64_t M = cfg->M, N = cfg->N, K = cfg->K;
   const int bs = cfg->bs;
   const int ncha = (int)enc_a_chunks(K), nchb = (int)enc_b_chunks(K);
-  char *w = static_cast<char *>(ws);
-  const size_t ra = (size_t)(M + M / bs), rb = (size_t)(N + N / bs);
-  double *pva = reinterpret_cast<double *>(w);
-  w += (ra * ncha * P * 8 + 255) / 256 * 256;
-  int *pia = reinterpret_cast<int *>(w);
-  w += (ra * ncha * P * 4 + 255) / 256 * 256;
-  double *pvb = reinterpret_cast<double *>(w);
-  w += (rb * nchb * P * 8 + 255) / 256 * 256;
-  int *pib = reinterpret_cast<int *>(w);
-  // top-p tables NULL: checksums only (the encoding of the fixed-eps and SEA comparators)
-  const bool tpa = A && out->topA_val, tpb = B && out->topB_val;
+  const EncWs e = enc_ws(cfg, ws);
+  // top-p tables NULL: checksums only (the encoding of the fixed-eps and SEA comparators);
+  // AABFT_FLAG_TOPP_IN_GEMM: the FP64 GEMM selects the top-p from its operand tiles instead
+  const bool defer = (cfg->flags & AABFT_FLAG_TOPP_IN_GEMM) && gemm_f64_topp_ok(cfg);
+  const bool tpa = A && out->topA_val && !defer, tpb = B && out->topB_val && !defer;
   if (A) {
-    dim3 grid(ncha, (unsigned)(M / bs));
+    const unsigned grid = (unsigned)((M / bs) * ncha);
     auto kern = tpa ? encode_a_kernel<T, P, true> : encode_a_kernel<T, P, false>;
-    kern<<<grid, 128, 0, st>>>(A, lda, K, bs, static_cast<T *>(out->Acs), out->ld_acs, pva, pia,
-                               ncha);
+    kern<<<grid, 128, 0, st>>>(A, lda, M, K, bs, static_cast<T *>(out->Acs), out->ld_acs, e.pva,
+                               e.pia, ncha);
     next_launch();
   }
   if (B) {
     const int NC = std::max(128, bs);
-    dim3 grid((unsigned)((N + NC - 1) / NC), nchb);
+    const unsigned grid = (unsigned)(((N + NC - 1) / NC) * nchb);
     if (NC == 128) {
       auto kern = tpb ? encode_b_kernel<T, P, 128, true> : encode_b_kernel<T, P, 128, false>;
-      kern<<<grid, 128, 0, st>>>(B, ldb, K, N, bs, static_cast<T *>(out->Bcs), out->ld_bcs, pvb,
-                                 pib, nchb);
+      kern<<<grid, 128, 0, st>>>(B, ldb, K, N, bs, static_cast<T *>(out->Bcs), out->ld_bcs, e.pvb,
+                                 e.pib, nchb);
     } else {
       auto kern = tpb ? encode_b_kernel<T, P, 256, true> : encode_b_kernel<T, P, 256, false>;
-      kern<<<grid, 256, 0, st>>>(B, ldb, K, N, bs, static_cast<T *>(out->Bcs), out->ld_bcs, pvb,
-                                 pib, nchb);
+      kern<<<grid, 256, 0, st>>>(B, ldb, K, N, bs, static_cast<T *>(out->Bcs), out->ld_bcs, e.pvb,
+                                 e.pib, nchb);
     }
     next_launch();
   }
   const int64_t nvec = (tpa ? M + M / bs : 0) + (tpb ? N + N / bs : 0);
   if (nvec > 0) {
-    topp_reduce_kernel<T, P><<<(unsigned)((nvec + 7) / 8), 256, 0, st>>>(
-        M, N, K, bs, pva, pia, ncha, pvb, pib, nchb, static_cast<const T *>(out->Acs),
-        out->ld_acs, static_cast<const T *>(out->Bcs), out->ld_bcs, out->topA_val,
-        out->topA_idx, out->topB_val, out->topB_idx, tpa, tpb);
+    topp_reduce_kernel<P><<<(unsigned)((nvec + 7) / 8), 256, 0, st>>>(
+        M, N, bs, e.pva, e.pia, ncha, e.pvb, e.pib, nchb, out->topA_val, out->topA_idx,
+        out->topB_val, out->topB_idx, tpa, tpb);
     next_launch();
   }
   return check_launch("aabft_encode");
@@ -343,9 +435,9 @@ aabft_status dispatch_p(const aabft_config *cfg, const void *A, int64_t lda, con
 size_t encode_ws_bytes(const aabft_config *cfg) {
   const size_t p = (size_t)cfg->p;
   const size_t ncha = (size_t)enc_a_chunks(cfg->K), nchb = (size_t)enc_b_chunks(cfg->K);
-  auto r = [](size_t b) { return (b + 255) / 256 * 256; };
   const size_t ra = (size_t)(cfg->M + cfg->M / cfg->bs), rb = (size_t)(cfg->N + cfg->N / cfg->bs);
-  return r(ra * ncha * p * 8) + r(ra * ncha * p * 4) + r(rb * nchb * p * 8) + r(rb * nchb * p * 4);
+  return r256e(ra * ncha * p * 8) + r256e(ra * ncha * p * 4) + r256e(rb * nchb * p * 8) +
+         r256e(rb * nchb * p * 4);
 }
 
 aabft_status launch_encode(const aabft_config *cfg, const void *A, int64_t lda, const void *B,

@@ -77,6 +77,7 @@ constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + BOOK +
 constexpr int GROUP_M = AABFT_F64_GROUP_M;
 constexpr int kMaxCtas = 1024;              // >= resident CTAs; sizes the split-K partial slots
 constexpr int ACC = MT * NT * 4;            // accumulators per thread
+constexpr int kTpMaxP = 4;                  // top-p selection in the GEMM for p <= 4
 
 struct GemmArgs {
   int64_t M, N, K, Mcs, Ncs;
@@ -100,6 +101,14 @@ struct GemmArgs {
   double *Rcol2;                      // BS = 64: partials of the wm = 1 warps (workspace)
   double *Rrow2;                      //          partials of the wn = 1 warps (workspace)
   int bs;
+  // top-p selection fused into the operand stream (TP > 0; DESIGN.md 6.1 "top-p in the GEMM")
+  double *topA_v;                     // (M + M/bs) x TP  final tables (aabft_encoded)
+  int *topA_i;
+  double *topB_v;                     // (N + N/bs) x TP
+  int *topB_i;
+  double *tp_v;                       // [kMaxCtas][128 lists][TP] stream-K partial lists
+  int *tp_i;
+  int *tp_flags;                      // [kMaxCtas]
 };
 
 struct Tile {
@@ -167,7 +176,177 @@ __device__ __forceinline__ double xor_bits(double v, uint64_t m) {
 
 // FAULTS: the Alg 3 injection instantiation (launched only with a fault list); the production
 // instantiation carries no fault bookkeeping in its k-loop.
-template <bool FAULTS>
+// ------------------------------------------------------------------ top-p in the GEMM
+// Step 1's top-p selection (Alg 1; the paper runs its global reduction "in
+// parallel to the matrix multiplication kernel", P:L320 / P:L368) taken from the operand
+// tiles the GEMM already streams through shared memory: the tiles of block-column 0 see every
+// row of A (type 0) and of Acs (type 1) over the whole K, the tiles of block-row 0 every
+// column of B (type 0) and of Bcs (type 2).  The TMA producer warp -- otherwise idle on the
+// empty barriers -- scans a stage kScanLag jobs after issuing it (the stage is refilled only
+// STAGES jobs later, by the same warp), lane l owning rows / columns l and l + 32.
+// MEASURED SLOWER than selecting in aabft_encode (the ~130 scanning CTAs
+// become stragglers, +0.35 ms on a 4.17 ms c2 GEMM against ~0.05 ms of top-p work in the
+// encode), so it is opt-in (AABFT_FLAG_TOPP_IN_GEMM) and ProtectedGemm leaves it off.  Within a segment k ascends, so the branch-free tp_push (new
+// element loses every tie) gives the sequential scan's list; stream-K partial lists are
+// parked like the accumulators and merged by the tile's owner with the full comparator.  No
+// extra HBM traffic; the encode stage keeps only the checksums.
+constexpr int kScanLag = STAGES - 1;  // measured best of 1..3 (tools/variants_time.sh)
+
+template <int P>
+struct TopScan {
+  int tile, kt0;
+  bool sa, sb;
+  Tile tl;
+  unsigned long long ka[2][P], kb[2][P];  // |value| bit patterns (integer-ALU selection)
+  double va[2][P], vb[2][P];              // values at the segment end (merge / store)
+  int ia[2][P], ib[2][P];
+};
+
+__device__ __forceinline__ void sk_owner_contributors_end(const GemmArgs &a, int tile, int64_t &it_end) {
+  it_end = (int64_t)(tile - a.waves * (int)gridDim.x + 1) * a.nk;
+}
+
+template <int P>
+__device__ __forceinline__ void tp_store(double *v_out, int *i_out, const double (&v)[P],
+                                         const int (&ix)[P]) {
+#pragma unroll
+  for (int r = 0; r < P; ++r) { v_out[r] = v[r]; i_out[r] = ix[r]; }
+}
+
+template <int P>
+__device__ __forceinline__ void tp_merge_from(double (&v)[P], int (&ix)[P], const double *sv,
+                                             const int *si) {
+#pragma unroll
+  for (int r = 0; r < P; ++r) tp_insert<P>(v, ix, __ldcg(sv + r), __ldcg(si + r));
+}
+
+template <int P>
+__device__ void scan_flush(const GemmArgs &a, TopScan<P> &sc, int kt_last, int lane) {
+  const bool first = sc.kt0 == 0, last = kt_last == a.nk - 1;
+#pragma unroll
+  for (int h = 0; h < 2; ++h)
+#pragma unroll
+    for (int r = 0; r < P; ++r) {  // empty slots keep the tp_init sentinel (-1.0, -1)
+      sc.va[h][r] = sc.ia[h][r] < 0 ? -1.0 : __longlong_as_double((long long)(sc.ka[h][r] - 1));
+      sc.vb[h][r] = sc.ib[h][r] < 0 ? -1.0 : __longlong_as_double((long long)(sc.kb[h][r] - 1));
+    }
+  if (!first) {  // stream-K contributor: park the partial lists, then signal the tile's owner
+    double *pv = a.tp_v + (int64_t)blockIdx.x * 128 * P;
+    int *pi = a.tp_i + (int64_t)blockIdx.x * 128 * P;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      if (sc.sa) tp_store<P>(pv + (lane + 32 * h) * P, pi + (lane + 32 * h) * P, sc.va[h], sc.ia[h]);
+      if (sc.sb) tp_store<P>(pv + (64 + lane + 32 * h) * P, pi + (64 + lane + 32 * h) * P, sc.vb[h], sc.ib[h]);
+    }
+    __threadfence();
+    __syncwarp();
+    if (lane == 0) atomicExch(&a.tp_flags[blockIdx.x], 1);
+    return;
+  }
+  if (!last) {  // owner of a split tile: merge the following CTAs' partial lists
+    int64_t it_end;
+    sk_owner_contributors_end(a, sc.tile, it_end);
+    for (int64_t c = blockIdx.x + 1; c < gridDim.x && sk_begin(a, c) < it_end; ++c) {
+      if (sk_begin(a, c + 1) == sk_begin(a, c)) continue;  // empty slice
+      if (lane == 0) {
+        while (atomicAdd(&a.tp_flags[c], 0) == 0) __nanosleep(64);
+        atomicExch(&a.tp_flags[c], 0);  // re-arm for the next launch
+        __threadfence();
+      }
+      __syncwarp();
+      const double *pv = a.tp_v + c * 128 * P;
+      const int *pi = a.tp_i + c * 128 * P;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        if (sc.sa) tp_merge_from<P>(sc.va[h], sc.ia[h], pv + (lane + 32 * h) * P, pi + (lane + 32 * h) * P);
+        if (sc.sb) tp_merge_from<P>(sc.vb[h], sc.ib[h], pv + (64 + lane + 32 * h) * P, pi + (64 + lane + 32 * h) * P);
+      }
+    }
+  }
+  // complete lists: data vectors first, then checksum vectors (aabft_encoded layout)
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    const int r = lane + 32 * h;
+    if (sc.sa) {
+      int64_t row = -1;
+      if (sc.tl.type == 0 && sc.tl.m0 + r < a.M) row = sc.tl.m0 + r;
+      if (sc.tl.type == 1 && sc.tl.m0 + r < a.Mcs) row = a.M + sc.tl.m0 + r;
+      if (row >= 0) tp_store<P>(a.topA_v + row * P, a.topA_i + row * P, sc.va[h], sc.ia[h]);
+    }
+    if (sc.sb) {
+      int64_t col = -1;
+      if (sc.tl.type == 0 && sc.tl.n0 + r < a.N) col = sc.tl.n0 + r;
+      if (sc.tl.type == 2 && sc.tl.n0 + r < a.Ncs) col = a.N + sc.tl.n0 + r;
+      if (col >= 0) tp_store<P>(a.topB_v + col * P, a.topB_i + col * P, sc.vb[h], sc.ib[h]);
+    }
+  }
+}
+
+template <int P>
+__device__ __forceinline__ void scan_job(const GemmArgs &a, const uint8_t *smem, uint64_t *full,
+                                         int js, int njobs, int64_t sk0, TopScan<P> &sc,
+                                         int lane) {
+  int tile, kt;
+  iter_of(a, js, sk0, tile, kt);
+  if (tile != sc.tile) {  // a new segment of consecutive k-tiles of one tile
+    sc.tile = tile;
+    sc.kt0 = kt;
+    sc.tl = tile_of(a, tile);
+    sc.sa = (sc.tl.type == 0 || sc.tl.type == 1) && sc.tl.n0 == 0;
+    sc.sb = (sc.tl.type == 0 || sc.tl.type == 2) && sc.tl.m0 == 0;
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+#pragma unroll
+      for (int r = 0; r < P; ++r) {  // key = |x| bits + 1, so the empty key 0 loses to |x| = 0
+        sc.ka[h][r] = 0ull; sc.kb[h][r] = 0ull; sc.ia[h][r] = -1; sc.ib[h][r] = -1;
+      }
+  }
+  if (sc.sa || sc.sb) {
+    const int s = js % STAGES;
+    mbar_wait(&full[s], (uint32_t)((js / STAGES) & 1));
+    const uint8_t *st = smem + s * STAGE_BYTES;
+    const int kbase = kt * BK;
+    const int lim = a.K - kbase < BK ? (int)(a.K - kbase) : BK;  // TMA zero-fills k >= K
+    if (sc.sa) {
+      // A tile: row r, column k at r*128 + ((k/2 ^ r%8) * 16) + (k%2)*8 (128B swizzle)
+#pragma unroll
+      for (int k = 0; k < BK; ++k) {
+        if (k < lim) {
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int r = lane + 32 * h;
+            const double x = *reinterpret_cast<const double *>(
+                st + r * 128 + ((((k >> 1) ^ (r & 7)) << 4) | ((k & 1) << 3)));
+            tp_push_bits<P>(sc.ka[h], sc.ia[h], abs_bits(x) + 1, kbase + k);
+          }
+        }
+      }
+    }
+    if (sc.sb) {
+      // B tile: 8 boxes of 8 columns; column c, row k at box*1024 + k*64 +
+      // (((c%8)/2 ^ (k/2)%4) * 16) + (c%2)*8 (64B swizzle)
+#pragma unroll
+      for (int k = 0; k < BK; ++k) {
+        if (k < lim) {
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int c = lane + 32 * h, cc = c & 7;
+            const double x = *reinterpret_cast<const double *>(
+                st + A_BYTES + (c >> 3) * 1024 + k * 64 +
+                ((((cc >> 1) ^ ((k >> 1) & 3)) << 4) | ((cc & 1) << 3)));
+            tp_push_bits<P>(sc.kb[h], sc.ib[h], abs_bits(x) + 1, kbase + k);
+          }
+        }
+      }
+    }
+  }
+  if (kt == a.nk - 1 || js == njobs - 1) {  // segment end
+    if (sc.sa || sc.sb) scan_flush<P>(a, sc, kt, lane);
+    sc.tile = -1;
+  }
+}
+
+template <bool FAULTS, int TP>
 __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
     gemm_f64_kernel(const __grid_constant__ CUtensorMap tmA,
                     const __grid_constant__ CUtensorMap tmAcs,
@@ -213,6 +392,9 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
     }
     int tile = -1, kt = 0;
     Tile tl{0, 0, 0};
+    constexpr int SP = TP > 0 ? TP : 1;
+    TopScan<SP> sc;
+    sc.tile = -1;
     for (int jn = 0; jn < njobs; ++jn) {
       if (tile < 0 || kt + 1 >= args.nk || jn == args.waves * args.nk) {
         iter_of(args, jn, sk0, tile, kt);
@@ -236,7 +418,11 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
         tma_load_2d(sa, tl.type == 1 ? &tmAcs : &tmA, &full[s], k, tl.m0);
       }
       __syncwarp();
+      if (TP > 0 && jn >= kScanLag) scan_job<SP>(args, smem, full, jn - kScanLag, njobs, sk0, sc, lane);
     }
+    if (TP > 0)
+      for (int js = max(0, njobs - kScanLag); js < njobs; ++js)
+        scan_job<SP>(args, smem, full, js, njobs, sk0, sc, lane);
     return;
   }
 
@@ -555,6 +741,17 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
   }
 }
 
+const void *kernel_for(bool faults, int tp) {
+  static const void *tab[2][kTpMaxP + 1] = {
+      {(const void *)gemm_f64_kernel<false, 0>, (const void *)gemm_f64_kernel<false, 1>,
+       (const void *)gemm_f64_kernel<false, 2>, (const void *)gemm_f64_kernel<false, 3>,
+       (const void *)gemm_f64_kernel<false, 4>},
+      {(const void *)gemm_f64_kernel<true, 0>, (const void *)gemm_f64_kernel<true, 1>,
+       (const void *)gemm_f64_kernel<true, 2>, (const void *)gemm_f64_kernel<true, 3>,
+       (const void *)gemm_f64_kernel<true, 4>}};
+  return tab[faults ? 1 : 0][tp];
+}
+
 PFN_cuTensorMapEncodeTiled_v12000 get_encoder() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
   if (!fn) {
@@ -594,9 +791,12 @@ bool make_map(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer, 
 }  // namespace
 
 static size_t r256z(size_t b) { return (b + 255) / 256 * 256; }
-static size_t red_off() {
-  return r256z((size_t)kMaxCtas * ACC * THREADS * sizeof(double) + kMaxCtas * sizeof(int));
-}
+// [split-K accumulator partials][flags][top-p flags][top-p partial values][indices][R planes]
+static size_t flags_off() { return r256z((size_t)kMaxCtas * ACC * THREADS * sizeof(double)); }
+static size_t tpv_off() { return flags_off() + r256z(2 * (size_t)kMaxCtas * sizeof(int)); }
+static size_t tpi_off() { return tpv_off() + r256z((size_t)kMaxCtas * 128 * kTpMaxP * sizeof(double)); }
+static size_t red_off() { return tpi_off() + r256z((size_t)kMaxCtas * 128 * kTpMaxP * sizeof(int)); }
+bool gemm_f64_topp_ok(const aabft_config *cfg) { return cfg->dtype == AABFT_F64 && cfg->p <= kTpMaxP; }
 size_t gemm_f64_ws_bytes(const aabft_config *cfg) {
   return red_off() + r256z((size_t)(cfg->M / cfg->bs) * cfg->N * 8 * (COL_PARTS - 1)) +
          r256z((size_t)cfg->M * (cfg->N / cfg->bs) * 8 * (ROW_PARTS - 1)) + 256;
@@ -625,20 +825,21 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
     int sms = 0, per_sm = 0;
     if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
       return check_launch("gemm_f64 SM count");
-    if (cudaFuncSetAttribute(gemm_f64_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             SMEM_BYTES) != cudaSuccess ||
-        cudaFuncSetAttribute(gemm_f64_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             SMEM_BYTES) != cudaSuccess)
-      return check_launch("gemm_f64 smem attribute");
-    int per_sm_f = 0;  // both instantiations must keep every CTA resident
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm_f, gemm_f64_kernel<true>, CTA_THREADS,
-                                                      SMEM_BYTES) != cudaSuccess)
-      return check_launch("gemm_f64 occupancy");
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, gemm_f64_kernel<false>, CTA_THREADS,
-                                                      SMEM_BYTES) != cudaSuccess || per_sm < 1)
-      return check_launch("gemm_f64 occupancy");
+    per_sm = 1 << 30;  // every instantiation must keep every CTA resident
+    for (int f = 0; f < 2; ++f)
+      for (int tp = 0; tp <= kTpMaxP; ++tp) {
+        const void *fn = kernel_for(f != 0, tp);
+        int n = 0;
+        if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES) !=
+            cudaSuccess)
+          return check_launch("gemm_f64 smem attribute");
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, CTA_THREADS, SMEM_BYTES) !=
+                cudaSuccess || n < 1)
+          return check_launch("gemm_f64 occupancy");
+        per_sm = std::min(per_sm, n);
+      }
     // every CTA must be resident (split-tile owners wait on later CTAs)
-    max_ctas = std::min(sms * std::min(per_sm, per_sm_f), kMaxCtas);
+    max_ctas = std::min(sms * per_sm, kMaxCtas);
     max_ctas_dev[dev & 63].store(max_ctas, std::memory_order_relaxed);
   }
   const int64_t M = cfg->M, N = cfg->N, K = cfg->K, bs = cfg->bs;
@@ -672,7 +873,17 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
   a.waves = waves;
   a.sk_iters = (ntiles - (int64_t)waves * grid) * nk;
   a.partials = static_cast<double *>(ws);
-  a.flags = reinterpret_cast<int *>(static_cast<char *>(ws) + (size_t)kMaxCtas * ACC * THREADS * sizeof(double));
+  a.flags = reinterpret_cast<int *>(static_cast<char *>(ws) + flags_off());
+  a.tp_flags = a.flags + kMaxCtas;
+  a.tp_v = reinterpret_cast<double *>(static_cast<char *>(ws) + tpv_off());
+  a.tp_i = reinterpret_cast<int *>(static_cast<char *>(ws) + tpi_off());
+  // top-p in the GEMM (aabft_config flag; FP64, p <= 4): the tables of `enc`
+  const int tp = (!plain && (cfg->flags & AABFT_FLAG_TOPP_IN_GEMM) && gemm_f64_topp_ok(cfg) &&
+                  enc->topA_val && enc->topB_val) ? cfg->p : 0;
+  a.topA_v = tp ? enc->topA_val : nullptr;
+  a.topA_i = tp ? enc->topA_idx : nullptr;
+  a.topB_v = tp ? enc->topB_val : nullptr;
+  a.topB_i = tp ? enc->topB_idx : nullptr;
   a.faults = faults;
   a.nfaults = faults ? nfaults : 0;
   a.bs = (int)bs;
@@ -697,12 +908,24 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
       return AABFT_EINVAL;
   }
   if (total > 0) {
-    if (a.sk_iters > 0 && cudaMemsetAsync(a.flags, 0, kMaxCtas * sizeof(int), st) != cudaSuccess)
+    if (a.sk_iters > 0 && cudaMemsetAsync(a.flags, 0, 2 * kMaxCtas * sizeof(int), st) != cudaSuccess)
       return check_launch("gemm_f64 flag reset");
-    if (a.nfaults > 0)
-      gemm_f64_kernel<true><<<grid, CTA_THREADS, SMEM_BYTES, st>>>(tA, tAcs, tB, tBcs, a);
-    else
-      gemm_f64_kernel<false><<<grid, CTA_THREADS, SMEM_BYTES, st>>>(tA, tAcs, tB, tBcs, a);
+    // split-tile owners spin on flags set by later CTAs: with a stream-K tail the launch is
+    // COOPERATIVE, so a grid that cannot be co-resident (other kernels, MPS, green contexts)
+    // waits for room or fails instead of hanging
+    cudaLaunchConfig_t lc = {};
+    lc.gridDim = dim3((unsigned)grid);
+    lc.blockDim = dim3(CTA_THREADS);
+    lc.dynamicSmemBytes = SMEM_BYTES;
+    lc.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;
+    attr[0].val.cooperative = a.sk_iters > 0 ? 1 : 0;
+    lc.attrs = attr;
+    lc.numAttrs = 1;
+    void *params[] = {&tA, &tAcs, &tB, &tBcs, &a};
+    cudaError_t e = cudaLaunchKernelExC(&lc, kernel_for(a.nfaults > 0, tp), params);
+    if (e != cudaSuccess) return check_launch("aabft_gemm(f64) launch");
     next_launch();
   }
   return check_launch("aabft_gemm(f64)");

@@ -20,10 +20,14 @@ def t(fn, reps=10):
         e0.record(); fn(); e1.record(); torch.cuda.synchronize(); ts.append(e0.elapsed_time(e1))
     return float(np.median(ts))
 tg = t(lambda: plan.gemm(A, B))
+def gemm_tp():
+    plan._topp_pending = True  # AABFT_FLAG_TOPP_IN_GEMM: the GEMM selects the top-p
+    plan.gemm(A, B)
+ttp = t(gemm_tp)
 tp = t(lambda: api.gemm_plain(A, B, out=Cp))
 tc = t(lambda: torch.matmul(A, B))
 fl = 2.0 * n ** 3
 aug = 2.0 * n * (n * n + 2 * (n // 64) * n)
 print(json.dumps({"lib": os.environ.get("AABFT_LIB", "default"), "n": n, "dtype": dt,
-                  "gemm_ms": tg, "gemm_aug_tflops": aug / tg / 1e9, "gemm_useful_tflops": fl / tg / 1e9,
+                  "gemm_ms": tg, "gemm_topp_ms": ttp, "gemm_topp_aug_tflops": aug / ttp / 1e9, "gemm_aug_tflops": aug / tg / 1e9, "gemm_useful_tflops": fl / tg / 1e9,
                   "plain_ms": tp, "plain_tflops": fl / tp / 1e9, "cublas_tflops": fl / tc / 1e9}))
