@@ -225,6 +225,12 @@ __device__ __forceinline__ void finish_block(const CheckArgs &a, int64_t blk, in
 // verdicts are gathered in shared memory (atomics only for the rare non-rounding checks) and
 // the device counters see one atomic per CTA.
 constexpr int kFusedThreads = 256;
+#ifndef AABFT_CHECK_EXP
+#define AABFT_CHECK_EXP 0
+#endif
+#ifndef AABFT_CHECK_CTAS
+#define AABFT_CHECK_CTAS 6
+#endif
 
 template <typename T, int P, bool EXT>
 __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a, BoundParams bp,
@@ -359,10 +365,12 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
     if (mr > 0.f) atomicMax(&s_mr, __float_as_uint(mr));
   }
   __syncthreads();
+#if AABFT_CHECK_EXP != 1
   if (tid < 8 && s_n[tid]) atomicAdd(reinterpret_cast<unsigned long long *>(a.cnt->n) + tid, s_n[tid]);
   if (tid == 8 && s_mr)
     atomicMax(reinterpret_cast<unsigned long long *>(&a.cnt->max_ratio),
               (unsigned long long)__double_as_longlong((double)__uint_as_float(s_mr)));
+#endif
 }
 
 // --------------------------------------------------------------------------- streaming check
@@ -587,7 +595,7 @@ aabft_status run_check(const aabft_config *cfg, const CheckArgs &a, BoundParams 
       const int JB = kFusedThreads / cfg->bs;
       const int64_t ngrp = (cfg->N / cfg->bs + JB - 1) / JB;
       const int64_t nunits = (cfg->M / cfg->bs) * ngrp;
-      const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(nunits, 148 * 6));
+      const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(nunits, 148 * AABFT_CHECK_CTAS));
       check_fused_kernel<T, P, EXT><<<grid, kFusedThreads, 0, st>>>(a, bp, nunits, (int)ngrp);
     } else if (cfg->bs <= 128) {
       dim3 grid((unsigned)((cfg->N + 127) / 128), (unsigned)(cfg->M / cfg->bs));
