@@ -58,7 +58,9 @@ def parse():
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="c2", choices=sorted(WORKLOADS))
+    ap.add_argument("--workload", default=None, choices=sorted(WORKLOADS),
+                    help="default: c2 (BASELINE configs[1]) at one GPU, c4 (configs[3], "
+                         "16384^2 row-sharded, strong scaling) with several")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--campaign", type=int, default=1, help="fault-injection runs (0 = skip)")
@@ -200,6 +202,8 @@ def run_reference(args, wl):
 # ------------------------------------------------------------------------------- our arm
 def main():
     args = parse()
+    if args.workload is None:
+        args.workload = "c2" if int(os.environ.get("WORLD_SIZE", "1")) == 1 else "c4"
     wl = dict(WORKLOADS[args.workload])
     if args.impl == "reference":
         return run_reference(args, wl)
@@ -236,23 +240,40 @@ def main():
                                             dtype=ndt)).to(dev)
     else:
         B = torch.empty(K, N, dtype=tdt, device=dev)
+    b_bcast_ms = None
     if world > 1:
+        # B replication: one broadcast from rank 0, timed on its own (not in the step: the
+        # operands are resident when the step starts)
         dist.broadcast(B, src=0)
-    plan = api.ProtectedGemm(m_local, N, K, dtype=tdt, bs=bs, p=P_TOPP, device=dev)
+        dist.barrier()
+        torch.cuda.synchronize(dev)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        dist.broadcast(B, src=0)
+        e1.record()
+        torch.cuda.synchronize(dev)
+        t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        b_bcast_ms = float(t[0])
+    from paper_conf_dsn_braunhw14_b200.distributed import ShardedProtectedGemm
+    sharded = (ShardedProtectedGemm(m_local, N, K, world=world, rank=rank, dtype=tdt, bs=bs,
+                                    p=P_TOPP, device=dev) if world > 1 else None)
+    plan = sharded.plan if sharded else api.ProtectedGemm(m_local, N, K, dtype=tdt, bs=bs,
+                                                          p=P_TOPP, device=dev)
     C_plain = torch.empty(m_local, N, dtype=tdt, device=dev)
     stream = torch.cuda.current_stream(dev)
-
-    from paper_conf_dsn_braunhw14_b200.distributed import reduce_counts
 
     graph = plan.capture(A, B) if (wl.get("graph") and world == 1) else None
 
     def step():
         if graph is not None:
             graph.replay()  # encode -> gemm -> check -> correct, one launch from the host
+        elif sharded is not None:
+            # encode of the local A rows and of this rank's B columns, all-gather of the B
+            # encoding, GEMM / check / correct of the local rows, counter all-reduce
+            sharded.run(A, B)
         else:
             plan.run(A, B)
-        if world > 1:
-            reduce_counts(plan.counts)  # the path's one exchange: SUM counters, MAX ratio
 
     in_bytes = (m_local * K + K * N) * (8 if wl['dtype'] == 'f64' else 4)
     flush = (torch.empty(256 << 20, dtype=torch.uint8, device=dev) if in_bytes < (126 << 20)
@@ -384,7 +405,9 @@ def main():
             "dtype": wl["dtype"], "data": "synthetic",
             "config": {"workload": wl["desc"], "M_per_rank": m_local, "M": M_glob, "N": N,
                        "K": K, "bs": bs, "p": P_TOPP, "recipe": wl["recipe"],
-                       "parallelism": f"row-sharded dp{world}",
+                       "parallelism": f"row-sharded dp{world}" + (
+                           ", B encoding sharded by columns + all-gather" if world > 1 else ""),
+                       "b_broadcast_ms": b_bcast_ms,
                        "cuda_graph": graph is not None,
                        "l2": ("inputs exceed L2 (A+B = %d MiB > 126 MB); no flush" % (in_bytes >> 20)
                               if flush is None else

@@ -32,6 +32,11 @@ def _worker(rank, world, port, q):
         c[8:9].view(torch.float64)[0] = [0.25, 7.5][rank]
         reduce_counts(c)
         q.put((rank, c[:8].tolist(), float(c[8:9].view(torch.float64)[0])))
+        # padded all-gather of unequal per-rank row counts (the sharded B encoding's exchange)
+        from paper_conf_dsn_braunhw14_b200.distributed import _all_gather_padded
+        x = torch.arange(3 * (rank + 1) * 2, dtype=torch.float64).reshape(3 * (rank + 1), 2) + 100 * rank
+        parts = _all_gather_padded(x, 6)
+        q.put(("G", rank, [p.tolist() for p in parts]))
         # B replication: broadcast from rank 0
         B = torch.arange(6, dtype=torch.float64) if rank == 0 else torch.zeros(6, dtype=torch.float64)
         dist.broadcast(B, src=0)
@@ -47,12 +52,16 @@ def test_counts_allreduce_gloo_world2():
     procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
     for p in procs:
         p.start()
-    out = [q.get(timeout=120) for _ in range(4)]
+    out = [q.get(timeout=120) for _ in range(6)]
     for p in procs:
         p.join(timeout=60)
         assert p.exitcode == 0
-    counts = [o for o in out if o[0] != "B"]
+    counts = [o for o in out if o[0] not in ("B", "G")]
     bs = [o for o in out if o[0] == "B"]
+    for _, rank, parts in [o for o in out if o[0] == "G"]:
+        for r, part in enumerate(parts):
+            exp = torch.arange(3 * (r + 1) * 2, dtype=torch.float64).reshape(3 * (r + 1), 2) + 100 * r
+            assert part == exp.tolist()
     assert len(counts) == 2
     for rank, n, mr in counts:
         assert n == [128, 63 + 62, 1, 1, 0, 16001, 6, 6]
