@@ -132,8 +132,10 @@ class ProtectedGemm:
         self.ldc = _pad_ld(N, dt)
         self.ld_ccol = _pad_ld(N, dt)
         self.ld_crow = _pad_ld(nJ, dt)
-        self._Acs = torch.empty(nI, self.ld_acs, dtype=dt, device=dev)
-        self._Bcs = torch.empty(K, self.ld_bcs, dtype=dt, device=dev)
+        # zeroed once: the 16-byte pitch padding is then defined for the FP32 GEMM's 16-byte
+        # cp.async row loads (compute-sanitizer initcheck clean; the padding never reaches C)
+        self._Acs = torch.zeros(nI, self.ld_acs, dtype=dt, device=dev)
+        self._Bcs = torch.zeros(K, self.ld_bcs, dtype=dt, device=dev)
         self._C = torch.empty(M, self.ldc, dtype=dt, device=dev)
         self._Ccol = torch.empty(nI, self.ld_ccol, dtype=dt, device=dev)
         self._Crow = torch.empty(M, self.ld_crow, dtype=dt, device=dev)

@@ -33,7 +33,9 @@ import synth  # noqa: E402
 from paper_conf_dsn_braunhw14_b200 import api  # noqa: E402
 
 WL = {"c2": (4096, 4096, 4096, 64, "f64", "uniform"), "c1": (128, 128, 128, 32, "f64", "uniform"),
-      "c3": (8192, 8192, 8192, 64, "f32", "wide"), "c2u100": (4096, 4096, 4096, 64, "f64", "uniform100")}
+      "c3": (8192, 8192, 8192, 64, "f32", "wide"), "c2u100": (4096, 4096, 4096, 64, "f64", "uniform100"),
+      # Eq 47 (Table IV / Fig 4's third workload): alpha = 0, kappa = 65536
+      "c2hdr": (4096, 4096, 4096, 64, "f64", "hdr65536")}
 
 
 def main():
@@ -50,8 +52,9 @@ def main():
     nbits = 64 if dts == "f64" else 32
     mant_bits = 52 if dts == "f64" else 23
 
-    A = torch.from_numpy(synth.generate(recipe, M, K, seed=1, matrix_id=0, dtype=ndt)).cuda()
-    B = torch.from_numpy(synth.generate(recipe, K, N, seed=2, matrix_id=1, dtype=ndt)).cuda()
+    from fig4 import make_input  # seeded recipes, or Eq 47 assembled on the device
+    A = make_input(recipe, M, K, 1, 0, ndt)
+    B = make_input(recipe, K, N, 2, 1, ndt)
     plan = api.ProtectedGemm(M, N, K, dtype=tdt, bs=bs, p=2)
     res = plan.run(A, B)
     torch.cuda.synchronize()

@@ -68,11 +68,26 @@ def flip_masks(rng, n, nflips, lo_bit, hi_bit):
     return m
 
 
+def make_input(recipe, rows, cols, seed, mid, ndt):
+    """Seeded inputs on the device.  'hdr<kappa>' is Eq 47 (Table IV; the paper's
+    third Fig 4 workload: alpha = 0, kappa = 65536), A = 10^alpha U D_kappa V^T
+    (reading R28) assembled on the device from the seeded host factors (input generation,
+    not the protected path)."""
+    if recipe.startswith("hdr"):
+        Ud, V = synth.hdr_factors(rows, cols, seed=seed, matrix_id=mid, kappa=float(recipe[3:]),
+                                  alpha=0.0)
+        X = torch.from_numpy(Ud).cuda() @ torch.from_numpy(V).cuda().T
+        return X.to(torch.float64 if ndt == np.float64 else torch.float32).contiguous()
+    return torch.from_numpy(synth.generate(recipe, rows, cols, seed=seed, matrix_id=mid,
+                                           dtype=ndt)).cuda()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--sizes", default="512,1024,2048,4096,8192")
-    ap.add_argument("--recipes", default="uniform,uniform100")
+    ap.add_argument("--recipes", default="uniform,uniform100,hdr65536",
+                    help="synth recipes, or hdr<kappa> for Eq 47 with alpha = 0")
     ap.add_argument("--bs", type=int, default=32)
     ap.add_argument("--reps", type=int, default=4, help="GEMMs per (size, site, flips) cell")
     ap.add_argument("--seed", type=int, default=11)
@@ -90,8 +105,8 @@ def main():
         for n in [int(v) for v in args.sizes.split(",")]:
             M = N = K = n
             bs = args.bs
-            A = torch.from_numpy(synth.generate(recipe, M, K, seed=1, matrix_id=0, dtype=ndt)).cuda()
-            B = torch.from_numpy(synth.generate(recipe, K, N, seed=2, matrix_id=1, dtype=ndt)).cuda()
+            A = make_input(recipe, M, K, 1, 0, ndt)
+            B = make_input(recipe, K, N, 2, 1, ndt)
             plan = api.ProtectedGemm(M, N, K, dtype=tdt, bs=bs, p=2)
             res = plan.run(A, B)
             torch.cuda.synchronize()

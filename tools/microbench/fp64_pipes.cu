@@ -95,16 +95,26 @@ __global__ void k_copy(const double4* __restrict__ a, double4* __restrict__ b, s
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) b[i] = a[i];
 }
 
+// best of `reps` timed launches; a launch that fails (e.g. too many registers for the block
+// size) returns -1 so no rate is printed for it (r01's impossible rows came from timing a
+// failed launch)
 template<class F>
 float time_it(F f, int reps) {
   cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
-  f(); cudaDeviceSynchronize();
+  f();
+  if (cudaGetLastError() != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess) return -1.f;
   float best = 1e30f;
   for (int r = 0; r < reps; ++r) {
-    cudaEventRecord(e0); f(); cudaEventRecord(e1); cudaEventSynchronize(e1);
+    cudaEventRecord(e0); f(); cudaEventRecord(e1);
+    if (cudaGetLastError() != cudaSuccess || cudaEventSynchronize(e1) != cudaSuccess) return -1.f;
     float ms; cudaEventElapsedTime(&ms, e0, e1); if (ms < best) best = ms;
   }
   return best;
+}
+
+void report(const char *kernel, int wpb, double flop, float ms) {
+  if (ms <= 0.f) printf("{\"kernel\":\"%s\",\"warps_per_block\":%d,\"tflops\":null,\"error\":\"launch failed\"}\n", kernel, wpb);
+  else printf("{\"kernel\":\"%s\",\"warps_per_block\":%d,\"tflops\":%.3f}\n", kernel, wpb, flop / (ms * 1e9));
 }
 
 int main() {
@@ -116,15 +126,15 @@ int main() {
     size_t warps = (size_t)blocks * wpb;
     float ms;
     ms = time_it([&] { k_m8n8k4<8><<<blocks, threads>>>(out, iters); }, 5);
-    printf("{\"kernel\":\"dmma_m8n8k4\",\"warps_per_block\":%d,\"tflops\":%.3f}\n", wpb, warps * iters * 8.0 * 512 / (ms * 1e9));
+    report("dmma_m8n8k4", wpb, warps * iters * 8.0 * 512, ms);
     ms = time_it([&] { k_m16n8k4<8><<<blocks, threads>>>(out, iters); }, 5);
-    printf("{\"kernel\":\"dmma_m16n8k4\",\"warps_per_block\":%d,\"tflops\":%.3f}\n", wpb, warps * iters * 8.0 * 1024 / (ms * 1e9));
+    report("dmma_m16n8k4", wpb, warps * iters * 8.0 * 1024, ms);
     ms = time_it([&] { k_m16n8k16<8><<<blocks, threads>>>(out, iters / 4); }, 5);
-    printf("{\"kernel\":\"dmma_m16n8k16\",\"warps_per_block\":%d,\"tflops\":%.3f}\n", wpb, warps * (iters / 4) * 8.0 * 4096 / (ms * 1e9));
+    report("dmma_m16n8k16", wpb, warps * (iters / 4) * 8.0 * 4096, ms);
     ms = time_it([&] { k_dfma<16><<<blocks, threads>>>(out, iters); }, 5);
-    printf("{\"kernel\":\"dfma\",\"warps_per_block\":%d,\"tflops\":%.3f}\n", wpb, warps * 32.0 * iters * 16 * 2 / (ms * 1e9));
+    report("dfma", wpb, warps * 32.0 * iters * 16 * 2, ms);
     ms = time_it([&] { k_ffma<16><<<blocks, threads>>>((float*)out, iters); }, 5);
-    printf("{\"kernel\":\"ffma\",\"warps_per_block\":%d,\"tflops\":%.3f}\n", wpb, warps * 32.0 * iters * 16 * 2 / (ms * 1e9));
+    report("ffma", wpb, warps * 32.0 * iters * 16 * 2, ms);
   }
   size_t bytes = (size_t)2 << 30; double4 *a, *b;
   CK(cudaMalloc(&a, bytes)); CK(cudaMalloc(&b, bytes)); cudaMemset(a, 0, bytes);
