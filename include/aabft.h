@@ -212,13 +212,20 @@ aabft_status aabft_gemm(const aabft_config *cfg, const void *A, int64_t lda, con
                         void *stream);
 
 /* Unprotected C = A.B with the same kernel family and scheduler (overhead denominator).
- * ws: device workspace of aabft_workspace_bytes(cfg) bytes (split-K partials). */
+ * ws: device workspace of aabft_gemm_plain_workspace_bytes(cfg) bytes (split-K partial
+ * slots and flags only; no checksum, top-p or reference-sum space).  Only cfg's dtype, M, N,
+ * K are used (bs and p must still validate). */
+size_t aabft_gemm_plain_workspace_bytes(const aabft_config *cfg);
 aabft_status aabft_gemm_plain(const aabft_config *cfg, const void *A, int64_t lda,
                               const void *B, int64_t ldb, void *C, int64_t ldc, void *ws,
                               size_t ws_bytes, void *stream);
 
 /* Step 3 (Alg 2; Eq 4-6).  Writes (M/bs)*(N/bs) reports and zeroes then fills
- * *counts (device).  Reference sums are sequential ascending in double (reading R11/R12). */
+ * *counts (device).  Reference sums are in double (reading R12): unfused (prod->Rcol/Rrow
+ * NULL, or FP32, or bs > 64) they re-sum C from memory in sequential ascending order -- the
+ * paper's check kernel; fused they are the GEMM epilogue's sums of the registers it
+ * stored (fixed shuffle-tree order, parity by tolerance) -- which sees every fault inside the
+ * GEMM (Alg 3) but not a corruption of C in memory after the store. */
 aabft_status aabft_check(const aabft_config *cfg, const aabft_encoded *enc,
                          const aabft_product *prod, aabft_block_report *reports,
                          aabft_counts *counts, void *ws, size_t ws_bytes, void *stream);

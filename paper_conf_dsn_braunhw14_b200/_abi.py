@@ -25,7 +25,7 @@ EXPORTED = ("aabft_workspace_bytes", "aabft_encode", "aabft_bound", "aabft_bound
             "aabft_gemm_plain", "aabft_check", "aabft_correct", "aabft_host_arena_bytes",
             "aabft_protected_gemm_host", "aabft_status_str", "aabft_last_error",
             "aabft_version", "aabft_launch_count", "aabft_checksum_errors", "aabft_sea_bound",
-            "aabft_check_ext", "aabft_correct_ext")
+            "aabft_check_ext", "aabft_correct_ext", "aabft_gemm_plain_workspace_bytes")
 
 
 class Config(C.Structure):
@@ -92,6 +92,8 @@ def lib():
         pc = C.POINTER(Config)
         L.aabft_workspace_bytes.argtypes = [pc]
         L.aabft_workspace_bytes.restype = sz
+        L.aabft_gemm_plain_workspace_bytes.argtypes = [pc]
+        L.aabft_gemm_plain_workspace_bytes.restype = sz
         L.aabft_host_arena_bytes.argtypes = [pc]
         L.aabft_host_arena_bytes.restype = sz
         L.aabft_encode.argtypes = [pc, vp, i64, vp, i64, C.POINTER(Encoded), vp, sz, vp]

@@ -369,7 +369,7 @@ def gemm_plain(A, B, out=None, stream=None):
     if out is None:
         out = torch.empty(M, _pad_ld(N, dt), dtype=dt, device=A.device)
     cfg = Config(_dtype_code(dt), 8, M, N, K, 1, 0, 3.0, 1, 0)  # bs=8: validation only
-    wsb = int(lib().aabft_workspace_bytes(C.byref(cfg)))
+    wsb = int(lib().aabft_gemm_plain_workspace_bytes(C.byref(cfg)))
     key = (A.device, wsb)
     if key not in _plain_ws:
         _plain_ws.clear()

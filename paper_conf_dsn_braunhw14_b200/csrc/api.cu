@@ -140,6 +140,11 @@ size_t aabft_workspace_bytes(const aabft_config *cfg) {
   return front_ws_bytes(cfg) + r256(gemm_ws_bytes(cfg)) + 256;
 }
 
+size_t aabft_gemm_plain_workspace_bytes(const aabft_config *cfg) {
+  if (validate(cfg) != AABFT_OK) return 0;
+  return cfg->dtype == AABFT_F64 ? r256(gemm_f64_plain_ws_bytes()) : 256;
+}
+
 aabft_status aabft_encode(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
                           int64_t ldb, const aabft_encoded *out, void *ws, size_t ws_bytes,
                           void *stream) {
@@ -226,8 +231,9 @@ static aabft_status gemm_common(const aabft_config *cfg, const void *A, int64_t 
                                 void *ws, size_t ws_bytes, void *stream) {
   aabft_status s = validate(cfg);
   if (s != AABFT_OK) return s;
-  if (!ws || ws_bytes < aabft_workspace_bytes(cfg)) {
-    set_error("workspace too small: need %zu bytes", aabft_workspace_bytes(cfg));
+  const size_t need = plain ? aabft_gemm_plain_workspace_bytes(cfg) : aabft_workspace_bytes(cfg);
+  if (!ws || ws_bytes < need) {
+    set_error("workspace too small: need %zu bytes", need);
     return AABFT_EWORKSPACE;
   }
   if (!A || !B || !out || !out->C) { set_error("gemm: A, B, C required"); return AABFT_EINVAL; }
@@ -250,7 +256,8 @@ static aabft_status gemm_common(const aabft_config *cfg, const void *A, int64_t 
   }
   if ((s = device_ok()) != AABFT_OK) return s;
   if (cfg->dtype == AABFT_F64)
-    return launch_gemm_f64(cfg, A, lda, B, ldb, enc, out, plain ? nullptr : faults, plain ? 0 : nfaults, plain, gemm_ws(cfg, ws), (cudaStream_t)stream);
+    return launch_gemm_f64(cfg, A, lda, B, ldb, enc, out, plain ? nullptr : faults, plain ? 0 : nfaults, plain,
+                           plain ? ws : gemm_ws(cfg, ws), (cudaStream_t)stream);
   return launch_gemm_f32(cfg, A, lda, B, ldb, enc, out, plain ? nullptr : faults, plain ? 0 : nfaults, plain, (cudaStream_t)stream);
 }
 

@@ -53,6 +53,7 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
 size_t encode_ws_bytes(const aabft_config *cfg);
 aabft_status launch_counts_sum(const aabft_counts *parts, int n, aabft_counts *out, cudaStream_t st);
 size_t gemm_f64_ws_bytes(const aabft_config *cfg);
+size_t gemm_f64_plain_ws_bytes();
 bool gemm_f64_topp_ok(const aabft_config *cfg);  // AABFT_FLAG_TOPP_IN_GEMM honoured
 void gemm_f64_red_ptrs(const aabft_config *cfg, void *gemm_ws, double **rcol2, double **rrow2);
 int gemm_f64_fused_parts(int bs, int *row_parts);  // returns column parts

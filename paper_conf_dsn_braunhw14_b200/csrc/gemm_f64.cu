@@ -798,9 +798,13 @@ static size_t tpi_off() { return tpv_off() + r256z((size_t)kMaxCtas * 128 * kTpM
 static size_t red_off() { return tpi_off() + r256z((size_t)kMaxCtas * 128 * kTpMaxP * sizeof(int)); }
 bool gemm_f64_topp_ok(const aabft_config *cfg) { return cfg->dtype == AABFT_F64 && cfg->p <= kTpMaxP; }
 size_t gemm_f64_ws_bytes(const aabft_config *cfg) {
+  // the fused reference-sum planes exist only where the fused check can run (bs <= 64)
+  if (cfg->bs > TILE) return red_off() + 256;
   return red_off() + r256z((size_t)(cfg->M / cfg->bs) * cfg->N * 8 * (COL_PARTS - 1)) +
          r256z((size_t)cfg->M * (cfg->N / cfg->bs) * 8 * (ROW_PARTS - 1)) + 256;
 }
+// the unprotected GEMM: split-K partial slots and flags only
+size_t gemm_f64_plain_ws_bytes() { return tpv_off() + 256; }
 int gemm_f64_fused_parts(int bs, int *row_parts) {
   *row_parts = bs > WTN ? bs / WTN : 1;
   return bs > 32 ? bs / 32 : 1;
