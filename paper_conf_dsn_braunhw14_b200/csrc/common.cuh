@@ -226,4 +226,15 @@ __device__ __forceinline__ void tma_load_2d(void *smem_dst, const CUtensorMap *t
       : "memory");
 }
 
+// 3D tiled TMA load global -> shared (complete_tx on an mbarrier)
+__device__ __forceinline__ void tma_load_3d(void *smem_dst, const CUtensorMap *tm, uint64_t *bar,
+                                            int c0, int c1, int c2) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(smem_u32(smem_dst)),
+      "l"(reinterpret_cast<uint64_t>(tm)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2)
+      : "memory");
+}
+
+
 }  // namespace aabft

@@ -38,14 +38,21 @@ namespace {
 #ifndef AABFT_F64_STAGES
 #define AABFT_F64_STAGES 4
 #endif
+#ifndef AABFT_F64_B3D
+#define AABFT_F64_B3D 0
+#endif
 #ifndef AABFT_F64_GROUP_M
 #define AABFT_F64_GROUP_M 16
 #endif
-constexpr int TILE = 64, BK = 16, STAGES = AABFT_F64_STAGES;
+#ifndef AABFT_F64_TN
+#define AABFT_F64_TN 64
+#endif
+constexpr int TM = 64, TN = AABFT_F64_TN, BK = 16, STAGES = AABFT_F64_STAGES;  // CTA tile TM x TN
+constexpr int TILE = TM;  // rows of a CTA tile (fused check: bs <= TILE)
 // B tiles as 4 TMA boxes of 16 columns x 16 k with the 128B swizzle (B16) instead of 8 boxes of
 // 8 columns with the 64B swizzle: half the copies per stage; needs its own k-permutation
 #ifndef AABFT_F64_B16
-#define AABFT_F64_B16 0
+#define AABFT_F64_B16 1
 #endif
 constexpr bool B16 = AABFT_F64_B16 != 0;
 #ifndef AABFT_F64_L2PROMO
@@ -57,7 +64,7 @@ constexpr bool B16 = AABFT_F64_B16 != 0;
 constexpr int NT = AABFT_F64_NT;            // n8 fragments per warp (warp tile 32 x 8*NT)
 constexpr int MT = 2;                       // m16 fragments per warp
 constexpr int WTN = NT * 8;                 // warp tile columns
-constexpr int WARPS_N = 64 / WTN;           // warps across the 64-column tile
+constexpr int WARPS_N = TN / WTN;           // warps across the tile's columns
 constexpr int NCW = 2 * WARPS_N;            // MMA warps per CTA (2 x WARPS_N)
 constexpr int THREADS = NCW * 32;           // MMA threads (named barrier 1)
 constexpr int CTA_THREADS = THREADS + 32;   // + 1 TMA producer warp
@@ -68,7 +75,7 @@ constexpr int CTAS_PER_SM = AABFT_F64_CTAS;  // 15 / 18 warps per SM (128 / <= 1
 constexpr int COL_PARTS = 2;                // fused column sums: BS=64 spans the 2 warp rows
 constexpr int ROW_PARTS = 64 / WTN;         // fused row sums: BS=64 spans WARPS_N warp columns
 constexpr int A_BYTES = TILE * BK * 8;      // 8 KiB
-constexpr int B_BYTES = BK * TILE * 8;      // 8 KiB
+constexpr int B_BYTES = BK * TN * 8;        // 8 KiB (TN 64) / 4 KiB (TN 32)
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 constexpr int MAXF = 64;                    // faults per 64x64 tile kept in smem (one per 8x8 block)
 constexpr int BOOK = 128;                   // barriers, counters, cursor
@@ -109,6 +116,7 @@ struct GemmArgs {
   double *tp_v;                       // [kMaxCtas][128 lists][TP] stream-K partial lists
   int *tp_i;
   int *tp_flags;                      // [kMaxCtas]
+  int b3d, bcs3d;                     // B / Bcs tiles as ONE 3-D TMA box (8 cols x 16 k x 8 groups)
 };
 
 struct Tile {
@@ -124,18 +132,18 @@ __device__ __forceinline__ Tile tile_of(const GemmArgs &a, int t) {
     const int first_m = g * GROUP_M;
     const int gm = min(a.tm0 - first_m, GROUP_M);
     const int in = t % group;
-    r.m0 = (first_m + in % gm) * TILE;
-    r.n0 = (in / gm) * TILE;
+    r.m0 = (first_m + in % gm) * TM;
+    r.n0 = (in / gm) * TN;
   } else if (t < a.n0 + a.n1) {
     t -= a.n0;
     r.type = 1;
-    r.m0 = (t / a.tn0) * TILE;
-    r.n0 = (t % a.tn0) * TILE;
+    r.m0 = (t / a.tn0) * TM;
+    r.n0 = (t % a.tn0) * TN;
   } else {
     t -= a.n0 + a.n1;
     r.type = 2;
-    r.m0 = (t / a.tn2) * TILE;
-    r.n0 = (t % a.tn2) * TILE;
+    r.m0 = (t / a.tn2) * TM;
+    r.n0 = (t % a.tn2) * TN;
   }
   return r;
 }
@@ -324,16 +332,19 @@ __device__ __forceinline__ void scan_job(const GemmArgs &a, const uint8_t *smem,
     }
     if (sc.sb) {
       // B tile: 8 boxes of 8 columns; column c, row k at box*1024 + k*64 +
-      // (((c%8)/2 ^ (k/2)%4) * 16) + (c%2)*8 (64B swizzle)
+      // (((c%8)/2 ^ (k/2)%4) * 16) + (c%2)*8 (64B swizzle), or the B16 layout
 #pragma unroll
       for (int k = 0; k < BK; ++k) {
         if (k < lim) {
 #pragma unroll
           for (int h = 0; h < 2; ++h) {
-            const int c = lane + 32 * h, cc = c & 7;
+            const int c = lane + 32 * h, cc = c & 7, c16 = c & 15;
+            // B16: 4 boxes of 16 columns, row k at box*2048 + k*128, 128B swizzle
             const double x = *reinterpret_cast<const double *>(
-                st + A_BYTES + (c >> 3) * 1024 + k * 64 +
-                ((((cc >> 1) ^ ((k >> 1) & 3)) << 4) | ((cc & 1) << 3)));
+                B16 ? st + A_BYTES + (c >> 4) * 2048 + k * 128 +
+                          ((((c16 >> 1) ^ (k & 7)) << 4) | ((c16 & 1) << 3))
+                    : st + A_BYTES + (c >> 3) * 1024 + k * 64 +
+                          ((((cc >> 1) ^ ((k >> 1) & 3)) << 4) | ((cc & 1) << 3)));
             tp_push_bits<P>(sc.kb[h], sc.ib[h], abs_bits(x) + 1, kbase + k);
           }
         }
@@ -344,6 +355,28 @@ __device__ __forceinline__ void scan_job(const GemmArgs &a, const uint8_t *smem,
     if (sc.sa || sc.sb) scan_flush<P>(a, sc, kt, lane);
     sc.tile = -1;
   }
+}
+
+// one stage of a job: expect the bytes, then the A box and the B tile (one 3-D box, or 2-D
+// boxes of 8 / 16 columns), all from the calling thread
+__device__ __forceinline__ void issue_stage(const GemmArgs &a, const CUtensorMap *tmA,
+                                            const CUtensorMap *tmAcs, const CUtensorMap *tmB,
+                                            const CUtensorMap *tmBcs, uint8_t *sa, uint64_t *bar,
+                                            const Tile &tl, int k) {
+  mbar_arrive_expect_tx(bar, STAGE_BYTES);
+  const CUtensorMap *mb = tl.type == 2 ? tmBcs : tmB;
+  if (!B16 && (tl.type == 2 ? a.bcs3d : a.b3d)) {
+    // the 8 column groups of the 64-column tile in one copy: smem [group][k][8 cols], the same
+    // bytes and 64B swizzle as 8 separate 2-D boxes
+    tma_load_3d(sa + A_BYTES, mb, bar, 0, k, tl.n0 / 8);
+  } else if (B16) {
+#pragma unroll
+    for (int b = 0; b < TN / 16; ++b) tma_load_2d(sa + A_BYTES + b * 2048, mb, bar, tl.n0 + b * 16, k);
+  } else {
+#pragma unroll
+    for (int b = 0; b < TN / 8; ++b) tma_load_2d(sa + A_BYTES + b * 1024, mb, bar, tl.n0 + b * 8, k);
+  }
+  tma_load_2d(sa, tl.type == 1 ? tmAcs : tmA, bar, k, tl.m0);
 }
 
 template <bool FAULTS, int TP>
@@ -406,17 +439,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
       if (jn >= STAGES) mbar_wait(&empty[s], (uint32_t)(((jn / STAGES) & 1) ^ 1));
       uint8_t *sa = smem + s * STAGE_BYTES;
       const int k = kt * BK;
-      if (lane == 0) mbar_arrive_expect_tx(&full[s], STAGE_BYTES);
-      __syncwarp();
-      if (B16 && lane < 4) {
-        tma_load_2d(sa + A_BYTES + lane * 2048, tl.type == 2 ? &tmBcs : &tmB, &full[s],
-                    tl.n0 + lane * 16, k);
-      } else if (!B16 && lane < 8) {
-        tma_load_2d(sa + A_BYTES + lane * 1024, tl.type == 2 ? &tmBcs : &tmB, &full[s],
-                    tl.n0 + lane * 8, k);
-      } else if (lane == 8) {
-        tma_load_2d(sa, tl.type == 1 ? &tmAcs : &tmA, &full[s], k, tl.m0);
-      }
+      if (lane == 0) issue_stage(args, &tmA, &tmAcs, &tmB, &tmBcs, sa, &full[s], tl, k);
       __syncwarp();
       if (TP > 0 && jn >= kScanLag) scan_job<SP>(args, smem, full, jn - kScanLag, njobs, sk0, sc, lane);
     }
@@ -478,7 +501,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
         else if (r >= args.M && c < args.N) { ftype = 1; r -= args.M; }
         else if (c >= args.N && r < args.M) { ftype = 2; c -= args.N; }
         else ftype = -1;
-        if (ftype == tl.type && r >= tl.m0 && r < tl.m0 + TILE && c >= tl.n0 && c < tl.n0 + TILE) {
+        if (ftype == tl.type && r >= tl.m0 && r < tl.m0 + TM && c >= tl.n0 && c < tl.n0 + TN) {
           const int slot = atomicAdd(s_nf, 1);
           if (slot < MAXF) {
             ft.row = r;
@@ -545,6 +568,9 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
       // release the stage to the producer (its last fragments were consumed by the ks = 3 DMMAs)
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[s]);
+#ifdef AABFT_F64_KSYNC
+      if ((kt & (AABFT_F64_KSYNC - 1)) == 0) mma_sync_bar();  // experiment: MMA warps in lockstep
+#endif
       if (FAULTS && nf > 0) {  // Alg 3 errorVecAdd1 at k-tile granularity
         for (int f = 0; f < nf; ++f) {
           const aabft_fault ft = s_f[f];
@@ -765,6 +791,22 @@ PFN_cuTensorMapEncodeTiled_v12000 get_encoder() {
   return fn;
 }
 
+// B as a 3-D tensor {8 columns, K rows, N/8 column groups} with strides {ldb, 8} elements: one
+// box {8, 16, 8} is a 64-column x 16-k tile laid out [group][k][col] (64B swizzle per 64-byte
+// row), i.e. exactly the 8 two-dimensional boxes of 8 columns.  Needs N % 8 == 0 (no group
+// straddles the row end).  Returns false (caller falls back to 2-D boxes) if not encodable.
+bool make_map_b3d(CUtensorMap *m, const void *base, uint64_t N, uint64_t K, uint64_t ld_elems) {
+  auto enc = get_encoder();
+  if (!enc || N % 8 != 0) return false;
+  cuuint64_t dims[3] = {8, K, N / 8};
+  cuuint64_t strides[2] = {ld_elems * 8, 64};
+  cuuint32_t box[3] = {8, BK, TN / 8};
+  cuuint32_t es[3] = {1, 1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, const_cast<void *>(base), dims, strides, box,
+             es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, AABFT_F64_L2PROMO,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 bool make_map(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer, uint64_t ld_elems,
               uint32_t box_inner, uint32_t box_outer, CUtensorMapSwizzle sw) {
   auto enc = get_encoder();
@@ -796,7 +838,9 @@ static size_t flags_off() { return r256z((size_t)kMaxCtas * ACC * THREADS * size
 static size_t tpv_off() { return flags_off() + r256z(2 * (size_t)kMaxCtas * sizeof(int)); }
 static size_t tpi_off() { return tpv_off() + r256z((size_t)kMaxCtas * 128 * kTpMaxP * sizeof(double)); }
 static size_t red_off() { return tpi_off() + r256z((size_t)kMaxCtas * 128 * kTpMaxP * sizeof(int)); }
-bool gemm_f64_topp_ok(const aabft_config *cfg) { return cfg->dtype == AABFT_F64 && cfg->p <= kTpMaxP; }
+bool gemm_f64_topp_ok(const aabft_config *cfg) {
+  return TN == 64 && cfg->dtype == AABFT_F64 && cfg->p <= kTpMaxP;  // producer-warp scan, 64-col tiles
+}
 size_t gemm_f64_ws_bytes(const aabft_config *cfg) {
   // the fused reference-sum planes exist only where the fused check can run (bs <= 64)
   if (cfg->bs > TILE) return red_off() + 256;
@@ -856,8 +900,8 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
   a.ld_ccol = plain ? 0 : out->ld_ccol;
   a.Crow = plain ? nullptr : static_cast<double *>(out->Crow);
   a.ld_crow = plain ? 0 : out->ld_crow;
-  const int64_t tm0 = (M + TILE - 1) / TILE, tn0 = (N + TILE - 1) / TILE;
-  const int64_t tm1 = (a.Mcs + TILE - 1) / TILE, tn2 = (a.Ncs + TILE - 1) / TILE;
+  const int64_t tm0 = (M + TM - 1) / TM, tn0 = (N + TN - 1) / TN;
+  const int64_t tm1 = (a.Mcs + TM - 1) / TM, tn2 = (a.Ncs + TN - 1) / TN;
   const int64_t ntiles = tm0 * tn0 + tm1 * tn0 + tm0 * tn2;
   const int64_t nk = (K + BK - 1) / BK;
   if (ntiles * nk >= ((int64_t)1 << 31) || M >= ((int64_t)1 << 31) || N >= ((int64_t)1 << 31)) {
@@ -898,18 +942,27 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
 
   CUtensorMap tA, tAcs, tB, tBcs;
   if (!make_map(&tA, A, K, M, lda, BK, TILE, CU_TENSOR_MAP_SWIZZLE_128B)) return AABFT_EINVAL;
-  if (!make_map(&tB, B, N, K, ldb, B16 ? 16 : 8, BK,
-                B16 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B))
+  a.b3d = a.bcs3d = 0;
+  if (AABFT_F64_B3D && !B16 && make_map_b3d(&tB, B, N, K, ldb)) {
+    a.b3d = 1;
+  } else if (!make_map(&tB, B, N, K, ldb, B16 ? 16 : 8, BK,
+                       B16 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B)) {
     return AABFT_EINVAL;
+  }
   if (plain) {
     tAcs = tA;
     tBcs = tB;
+    a.bcs3d = a.b3d;
   } else {
     if (!make_map(&tAcs, enc->Acs, K, a.Mcs, enc->ld_acs, BK, TILE, CU_TENSOR_MAP_SWIZZLE_128B))
       return AABFT_EINVAL;
-    if (!make_map(&tBcs, enc->Bcs, a.Ncs, K, enc->ld_bcs, B16 ? 16 : 8, BK,
-                  B16 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B))
+    if (AABFT_F64_B3D && !B16 &&
+        make_map_b3d(&tBcs, enc->Bcs, (uint64_t)a.Ncs, K, enc->ld_bcs)) {
+      a.bcs3d = 1;
+    } else if (!make_map(&tBcs, enc->Bcs, a.Ncs, K, enc->ld_bcs, B16 ? 16 : 8, BK,
+                         B16 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B)) {
       return AABFT_EINVAL;
+    }
   }
   if (total > 0) {
     if (a.sk_iters > 0 && cudaMemsetAsync(a.flags, 0, 2 * kMaxCtas * sizeof(int), st) != cudaSuccess)
