@@ -75,23 +75,24 @@ __device__ __forceinline__ void kp_push(KT (&v)[P], int (&ix)[P], KT a, int idx)
   ix[0] = g[0] ? idx : ix[0];
 }
 
-// insertion with the full order (key desc, index asc; empty slots have index -1 and key 0)
+// insertion with the full order (key desc, index asc; empty slots: key 0, index -1, which as
+// an unsigned index is larger than every real one).  Branch-free: g[r] = "a precedes slot r"
+// is monotone in r for a sorted list, so the same shift as kp_push applies; an empty candidate
+// (key 0, index -1) precedes nothing.
 template <int P, typename KT>
 __device__ __forceinline__ void kp_insert(KT (&v)[P], int (&ix)[P], KT a, int idx) {
-  if (idx < 0) return;
+  bool g[P];
 #pragma unroll
-  for (int r = 0; r < P; ++r) {
-    const bool better = a > v[r] || (a == v[r] && (ix[r] < 0 || idx < ix[r]));
-    if (better) {
-      const KT tv = v[r];
-      const int ti = ix[r];
-      v[r] = a;
-      ix[r] = idx;
-      a = tv;
-      idx = ti;
-      if (idx < 0) break;
-    }
+  for (int r = 0; r < P; ++r) g[r] = a > v[r] || (a == v[r] && (unsigned)idx < (unsigned)ix[r]);
+#pragma unroll
+  for (int r = P - 1; r >= 1; --r) {
+    const KT vr = g[r - 1] ? v[r - 1] : (g[r] ? a : v[r]);
+    const int ir = g[r - 1] ? ix[r - 1] : (g[r] ? idx : ix[r]);
+    v[r] = vr;
+    ix[r] = ir;
   }
+  v[0] = g[0] ? a : v[0];
+  ix[0] = g[0] ? idx : ix[0];
 }
 
 template <int P, typename KT>
@@ -136,17 +137,23 @@ __device__ __forceinline__ void merge_vector(const double *__restrict__ pv, cons
 
 // ---------------------------------------------------------------------------------- A
 // 1-D grid: unit u -> block-row I = u / nch, column chunk = u % nch (128 columns); 128 threads.
+template <typename T>
+__host__ __device__ constexpr int enc_a_smem() { return kStrip * (kEncAChunk + 4) * (int)sizeof(typename Key<T>::type); }
+template <typename T, int NC>
+__host__ __device__ constexpr int enc_b_smem() { return ((NC * sizeof(T) > 1024) ? 16 : kStrip) * (NC + 1) * (int)sizeof(T); }
+
 template <typename T, int P, bool TOPP>
-__global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, int64_t lda,
-                                                       int64_t M, int64_t K, int bs,
-                                                       T *__restrict__ Acs, int64_t ld_acs,
-                                                       double *__restrict__ pv,
-                                                       int *__restrict__ pi, int nch) {
+__device__ __forceinline__ void encode_a_body(const T *__restrict__ A, int64_t lda, int64_t M,
+                                              int64_t K, int bs, T *__restrict__ Acs,
+                                              int64_t ld_acs, double *__restrict__ pv,
+                                              int *__restrict__ pi, int nch, unsigned unit,
+                                              unsigned char *sbuf) {
   using KT = typename Key<T>::type;
-  __shared__ KT tile[kStrip][kEncAChunk + 4];  // keys of |A| strip; conflict-free lane reads
+  // keys of the |A| strip, stride kEncAChunk + 4: conflict-free lane reads
+  KT (*tile)[kEncAChunk + 4] = reinterpret_cast<KT (*)[kEncAChunk + 4]>(sbuf);
   const int c = threadIdx.x;
-  const int chunk = (int)(blockIdx.x % (unsigned)nch);
-  const int64_t I = blockIdx.x / (unsigned)nch;
+  const int chunk = (int)(unit % (unsigned)nch);
+  const int64_t I = unit / (unsigned)nch;
   const int64_t k = (int64_t)chunk * kEncAChunk + c;
   const bool kin = k < K;
   const int r = c >> 2, q = c & 3;  // top-p role: row r of the strip, column phase q
@@ -177,19 +184,25 @@ __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, 
     if (r0 + kStrip < bs) load_strip(r0 + kStrip);
     if (!TOPP) continue;  // checksums only (fixed-eps / SEA ABFT comparators, NEXT-3)
     __syncthreads();
-    KT v[P];
-    int ix[P];
+    KT v[P], v2[P];
+    int ix[P], ix2[P];
     kp_init<P>(v, ix);
+    kp_init<P>(v2, ix2);
     if (r < rows) {
-      // ascending columns into this lane's own list: the new element loses every tie
+      // ascending columns into this lane's own two lists (columns q + 8t and q + 4 + 8t: two
+      // independent dependency chains): the new element loses every tie within its list
       const int kbase = chunk * kEncAChunk;
       const int lim = K - kbase < kEncAChunk ? (int)(K - kbase) : kEncAChunk;
       const KT *trow = tile[r];
-#pragma unroll 8
-      for (int cc = q; cc < kEncAChunk; cc += 4) {
-        const KT key = cc < lim ? trow[cc] : KT(0);  // key 0 never enters the list
-        kp_push<P, KT>(v, ix, key, kbase + cc);
+#pragma unroll 4
+      for (int cc = q; cc < kEncAChunk; cc += 8) {
+        const KT k1 = cc < lim ? trow[cc] : KT(0);  // key 0 never enters a list
+        const KT k2 = cc + 4 < lim ? trow[cc + 4] : KT(0);
+        kp_push<P, KT>(v, ix, k1, kbase + cc);
+        kp_push<P, KT>(v2, ix2, k2, kbase + cc + 4);
       }
+#pragma unroll
+      for (int t = 0; t < P; ++t) kp_insert<P, KT>(v, ix, v2[t], ix2[t]);
     }
     kp_shfl_merge<P, KT>(v, ix, 1);
     kp_shfl_merge<P, KT>(v, ix, 2);
@@ -226,32 +239,52 @@ __global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, 
   }
 }
 
+template <typename T, int P, bool TOPP>
+__global__ void __launch_bounds__(128) encode_a_kernel(const T *__restrict__ A, int64_t lda,
+                                                       int64_t M, int64_t K, int bs,
+                                                       T *__restrict__ Acs, int64_t ld_acs,
+                                                       double *__restrict__ pv,
+                                                       int *__restrict__ pi, int nch) {
+  __shared__ __align__(16) unsigned char sbuf[enc_a_smem<T>()];
+  encode_a_body<T, P, TOPP>(A, lda, M, K, bs, Acs, ld_acs, pv, pi, nch, blockIdx.x, sbuf);
+}
+
 // ---------------------------------------------------------------------------------- B
 // 1-D grid: unit u -> column chunk jc = u / nch (NC columns), row chunk kc = u % nch
 // (kEncBChunk rows of B); NC threads (NC = max(128, bs)).
 template <typename T, int P, int NC, bool TOPP>
-__global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, int64_t ldb,
-                                                      int64_t K, int64_t N, int bs,
-                                                      T *__restrict__ Bcs, int64_t ld_bcs,
-                                                      double *__restrict__ pv,
-                                                      int *__restrict__ pi, int nch) {
+__device__ __forceinline__ void encode_b_body(const T *__restrict__ B, int64_t ldb, int64_t K,
+                                              int64_t N, int bs, T *__restrict__ Bcs,
+                                              int64_t ld_bcs, double *__restrict__ pv,
+                                              int *__restrict__ pi, int nch, unsigned unit,
+                                              unsigned char *sbuf) {
   using KT = typename Key<T>::type;
   constexpr int SB = (NC * sizeof(T) > 1024) ? 16 : kStrip;  // strip rows (smem <= 48 KiB)
-  __shared__ T tile[SB][NC + 1];  // odd stride -> conflict-free per-row sequential reads
+  // odd stride NC + 1: conflict-free per-row sequential reads
+  T (*tile)[NC + 1] = reinterpret_cast<T (*)[NC + 1]>(sbuf);
   const int c = threadIdx.x;
-  const int64_t jc = blockIdx.x / (unsigned)nch;
-  const int kc = (int)(blockIdx.x % (unsigned)nch);
+  const int64_t jc = unit / (unsigned)nch;
+  const int kc = (int)(unit % (unsigned)nch);
   const int64_t j = jc * NC + c;
   const bool jin = j < N;
   const int64_t kbeg = (int64_t)kc * kEncBChunk;
   const int64_t kend = K < kbeg + kEncBChunk ? K : kbeg + kEncBChunk;
   const int nblk = NC / bs;  // checksum blocks covered by this CTA (<= 16)
+  // checksum-column top-p.  bs >= 32 (at most one block per warp): a running list per lane --
+  // lane rr of the warp owning block jb sees rows k0 + rr in ascending k across strips --
+  // merged across the warp once at the end.  Smaller blocks (several per warp): the strip's
+  // 32 row sums are folded into a shared-memory list per block after every strip.
+  const bool lane_lists = nblk <= NC / 32;
+  KT cvl[P];
+  int cil[P];
+  kp_init<P>(cvl, cil);
   __shared__ KT s_cv[16][P];
   __shared__ int s_ci[16][P];
   if (c < 16 * P) { s_cv[c / P][c % P] = 0; s_ci[c / P][c % P] = -1; }
-  KT v[P];
-  int ix[P];
+  KT v[P], v2[P];  // running top-p of column j over even / odd rows (two dependency chains)
+  int ix[P], ix2[P];
   kp_init<P>(v, ix);
+  kp_init<P>(v2, ix2);
   // register double buffering as in encode A: strip k0 + SB is loaded during the row sums
   T vals[SB];
   auto load_strip = [&](int64_t k0) {
@@ -274,14 +307,20 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
       for (int rr = 0; rr < SB; ++rr) {
         tile[rr][c] = vals[rr];
         // ascending k, own list: the new element loses every tie
-        if (TOPP) kp_push<P, KT>(v, ix, Key<T>::of(vals[rr]), k0i + rr);
+        if (TOPP) {
+          if (rr & 1) kp_push<P, KT>(v2, ix2, Key<T>::of(vals[rr]), k0i + rr);
+          else kp_push<P, KT>(v, ix, Key<T>::of(vals[rr]), k0i + rr);
+        }
       }
     } else {
 #pragma unroll
       for (int rr = 0; rr < SB; ++rr) {
         if (rr < rows) {
           tile[rr][c] = vals[rr];
-          if (TOPP) kp_push<P, KT>(v, ix, Key<T>::of(vals[rr]), k0i + rr);
+          if (TOPP) {
+            if (rr & 1) kp_push<P, KT>(v2, ix2, Key<T>::of(vals[rr]), k0i + rr);
+            else kp_push<P, KT>(v, ix, Key<T>::of(vals[rr]), k0i + rr);
+          }
         }
       }
     }
@@ -300,9 +339,12 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
         T sm = T(0);
         for (int jj = 0; jj < bs; ++jj) sm = sm + tile[rr][jb * bs + jj];
         Bcs[(k0 + rr) * ld_bcs + J] = sm;
-        if (TOPP) kp_push<P, KT>(lv, li, Key<T>::of(sm), (int)(k0 + rr));
+        if (TOPP) {
+          if (lane_lists) kp_push<P, KT>(cvl, cil, Key<T>::of(sm), (int)(k0 + rr));
+          else kp_push<P, KT>(lv, li, Key<T>::of(sm), (int)(k0 + rr));
+        }
       }
-      if (!TOPP) continue;
+      if (!TOPP || lane_lists) continue;
 #pragma unroll
       for (int m = 16; m >= 1; m >>= 1) kp_shfl_merge<P, KT>(lv, li, m);
       if (rr == 0) {
@@ -315,7 +357,19 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
     __syncthreads();
   }
   if (!TOPP) return;
-  if (c < nblk && (jc * nblk + c) * bs < N) {
+#pragma unroll
+  for (int t = 0; t < P; ++t) kp_insert<P, KT>(v, ix, v2[t], ix2[t]);
+  if (lane_lists) {
+    // checksum columns: merge the 32 lanes' lists of the warp's block once
+    const int jb = c >> 5;
+    if (jb < nblk) {  // warp-uniform
+#pragma unroll
+      for (int m = 16; m >= 1; m >>= 1) kp_shfl_merge<P, KT>(cvl, cil, m);
+      const int64_t J = jc * nblk + jb;
+      if ((c & 31) == 0 && J * bs < N)
+        kp_store<T, P>(pv + ((N + J) * nch + kc) * P, pi + ((N + J) * nch + kc) * P, cvl, cil);
+    }
+  } else if (c < nblk && (jc * nblk + c) * bs < N) {
     const int64_t J = jc * nblk + c;
     KT cv[P];
     int ci[P];
@@ -324,6 +378,33 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
     kp_store<T, P>(pv + ((N + J) * nch + kc) * P, pi + ((N + J) * nch + kc) * P, cv, ci);
   }
   if (jin) kp_store<T, P>(pv + (j * nch + kc) * P, pi + (j * nch + kc) * P, v, ix);
+}
+
+template <typename T, int P, int NC, bool TOPP>
+__global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, int64_t ldb,
+                                                      int64_t K, int64_t N, int bs,
+                                                      T *__restrict__ Bcs, int64_t ld_bcs,
+                                                      double *__restrict__ pv,
+                                                      int *__restrict__ pi, int nch) {
+  __shared__ __align__(16) unsigned char sbuf[enc_b_smem<T, NC>()];
+  encode_b_body<T, P, NC, TOPP>(B, ldb, K, N, bs, Bcs, ld_bcs, pv, pi, nch, blockIdx.x, sbuf);
+}
+
+// A and B in ONE launch (bs <= 128): the B units (longer: kEncBChunk rows each) come first,
+// then the A units; one shared buffer serves whichever body the CTA runs.  Saves a launch
+// boundary and lets the A units fill the machine while B's last units finish.
+template <typename T, int P, bool TOPP>
+__global__ void __launch_bounds__(128) encode_ab_kernel(
+    const T *__restrict__ A, int64_t lda, int64_t M, int64_t K, int bs, T *__restrict__ Acs,
+    int64_t ld_acs, double *__restrict__ pva, int *__restrict__ pia, int ncha,
+    const T *__restrict__ B, int64_t ldb, int64_t N, T *__restrict__ Bcs, int64_t ld_bcs,
+    double *__restrict__ pvb, int *__restrict__ pib, int nchb, unsigned nB) {
+  constexpr int SA = enc_a_smem<T>(), SBb = enc_b_smem<T, 128>();
+  __shared__ __align__(16) unsigned char sbuf[SA > SBb ? SA : SBb];
+  if (blockIdx.x < nB)
+    encode_b_body<T, P, 128, TOPP>(B, ldb, K, N, bs, Bcs, ld_bcs, pvb, pib, nchb, blockIdx.x, sbuf);
+  else
+    encode_a_body<T, P, TOPP>(A, lda, M, K, bs, Acs, ld_acs, pva, pia, ncha, blockIdx.x - nB, sbuf);
 }
 
 // ---------------------------------------------------------------------------------- step 3
@@ -380,6 +461,17 @@ aabft_status run_encode(const aabft_config *cfg, const T *A, int64_t lda, const 
   // AABFT_FLAG_TOPP_IN_GEMM: the FP64 GEMM selects the top-p from its operand tiles instead
   const bool defer = (cfg->flags & AABFT_FLAG_TOPP_IN_GEMM) && gemm_f64_topp_ok(cfg);
   const bool tpa = A && out->topA_val && !defer, tpb = B && out->topB_val && !defer;
+  const int NCb = std::max(128, bs);
+  if (A && B && NCb == 128 && tpa == tpb) {
+    const unsigned nA = (unsigned)((M / bs) * ncha), nB = (unsigned)(((N + 127) / 128) * nchb);
+    auto kern = tpa ? encode_ab_kernel<T, P, true> : encode_ab_kernel<T, P, false>;
+    kern<<<nA + nB, 128, 0, st>>>(A, lda, M, K, bs, static_cast<T *>(out->Acs), out->ld_acs, e.pva,
+                                  e.pia, ncha, B, ldb, N, static_cast<T *>(out->Bcs), out->ld_bcs,
+                                  e.pvb, e.pib, nchb, nB);
+    next_launch();
+    A = nullptr;  // both done
+    B = nullptr;
+  }
   if (A) {
     const unsigned grid = (unsigned)((M / bs) * ncha);
     auto kern = tpa ? encode_a_kernel<T, P, true> : encode_a_kernel<T, P, false>;

@@ -17,6 +17,9 @@ def t(fn, reps=20):
     ts = []
     for _ in range(reps):
         e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+        # keep the GPU busy while the host enqueues, so the events bracket device time only
+        # (on an idle stream e0 completes at once and the host's launch latency is counted)
+        torch.cuda._sleep(2_000_000)
         e0.record(); fn(); e1.record(); torch.cuda.synchronize(); ts.append(e0.elapsed_time(e1))
     return float(np.median(ts)) * 1e3
 out = {"lib": os.environ.get("AABFT_LIB", "default"), "n": n, "dtype": dt,
