@@ -225,9 +225,6 @@ __device__ __forceinline__ void finish_block(const CheckArgs &a, int64_t blk, in
 // verdicts are gathered in shared memory (atomics only for the rare non-rounding checks) and
 // the device counters see one atomic per CTA.
 constexpr int kFusedThreads = 256;
-#ifndef AABFT_CHECK_EXP
-#define AABFT_CHECK_EXP 0
-#endif
 #ifndef AABFT_CHECK_CTAS
 #define AABFT_CHECK_CTAS 6
 #endif
@@ -304,8 +301,13 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
         }
         r = (float)ratio_fast(d, bc.eps);
       }
-      for (int m = 1; m < cseg; m <<= 1) r = fmaxf(r, __shfl_xor_sync(0xffffffffu, r, m));
-      if ((lane & (cseg - 1)) == 0 && r > 0.f) atomicMax(&s_rmax[Jc], __float_as_uint(r));
+      unsigned rb = __float_as_uint(r);  // r >= 0: bit order == value order
+      if (cseg == 32) {
+        rb = __reduce_max_sync(0xffffffffu, rb);
+      } else {
+        for (int m = 1; m < cseg; m <<= 1) rb = max(rb, __shfl_xor_sync(0xffffffffu, rb, m));
+      }
+      if ((lane & (cseg - 1)) == 0 && rb) atomicMax(&s_rmax[Jc], rb);
     }
     {
       float r = 0.f;
@@ -319,8 +321,9 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
         }
         r = (float)ratio_fast(d, brw.eps);
       }
-      for (int m = JB; m < 32; m <<= 1) r = fmaxf(r, __shfl_xor_sync(0xffffffffu, r, m));
-      if (lane < JB && r > 0.f) atomicMax(&s_rmax[Jr], __float_as_uint(r));
+      unsigned rb = __float_as_uint(r);
+      for (int m = JB; m < 32; m <<= 1) rb = max(rb, __shfl_xor_sync(0xffffffffu, rb, m));
+      if (lane < JB && rb) atomicMax(&s_rmax[Jr], rb);
     }
     __syncthreads();
     // ---- block verdicts (warp 0: JB <= 32 blocks)
@@ -350,27 +353,24 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
     }
     __syncthreads();  // the per-block slots are re-initialised by the next unit
   }
-  // ---- CTA aggregation: one global atomic per non-zero counter
+  // ---- CTA aggregation: warp reductions (REDUX), then one global atomic per non-zero counter
+  // (per-thread totals are far below 2^32: a CTA handles a few units of 2 x 256 checks)
   my_n[5] = cls_tot[0]; my_n[6] = cls_tot[1]; my_n[7] = cls_tot[2];
+  unsigned wn[8];
 #pragma unroll
-  for (int c = 0; c < 8; ++c) {
-#pragma unroll
-    for (int m = 16; m >= 1; m >>= 1) my_n[c] += __shfl_xor_sync(0xffffffffu, my_n[c], m);
-  }
-#pragma unroll
-  for (int m = 16; m >= 1; m >>= 1) mr = fmaxf(mr, __shfl_xor_sync(0xffffffffu, mr, m));
+  for (int c = 0; c < 8; ++c) wn[c] = __reduce_add_sync(0xffffffffu, (unsigned)my_n[c]);
+  const unsigned wmr = __reduce_max_sync(0xffffffffu, __float_as_uint(mr));
   if (lane == 0) {
+#pragma unroll
     for (int c = 0; c < 8; ++c)
-      if (my_n[c]) atomicAdd(&s_n[c], my_n[c]);
-    if (mr > 0.f) atomicMax(&s_mr, __float_as_uint(mr));
+      if (wn[c]) atomicAdd(&s_n[c], (unsigned long long)wn[c]);
+    if (wmr) atomicMax(&s_mr, wmr);
   }
   __syncthreads();
-#if AABFT_CHECK_EXP != 1
   if (tid < 8 && s_n[tid]) atomicAdd(reinterpret_cast<unsigned long long *>(a.cnt->n) + tid, s_n[tid]);
   if (tid == 8 && s_mr)
     atomicMax(reinterpret_cast<unsigned long long *>(&a.cnt->max_ratio),
               (unsigned long long)__double_as_longlong((double)__uint_as_float(s_mr)));
-#endif
 }
 
 // --------------------------------------------------------------------------- streaming check

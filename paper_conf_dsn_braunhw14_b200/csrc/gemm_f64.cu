@@ -72,15 +72,20 @@ constexpr int CTA_THREADS = THREADS + 32;   // + 1 TMA producer warp
 #define AABFT_F64_CTAS (NCW == 4 ? 3 : 2)
 #endif
 constexpr int CTAS_PER_SM = AABFT_F64_CTAS;  // 15 / 18 warps per SM (128 / <= 102 registers)
-constexpr int COL_PARTS = 2;                // fused column sums: BS=64 spans the 2 warp rows
-constexpr int ROW_PARTS = 64 / WTN;         // fused row sums: BS=64 spans WARPS_N warp columns
+// BS = 64 on a 64 x 64 tile of 2 x 2 warps: the block is the CTA tile, and the epilogue
+// completes its column / row reference sums inside the CTA (shared memory, one barrier) --
+// otherwise a block larger than a warp tile leaves per-warp "parts" in the workspace
+constexpr bool kCtaSums = TM == 64 && TN == 64 && WTN == 32;
+constexpr int COL_PARTS = kCtaSums ? 1 : 2;           // fused column sums of a BS = 64 block
+constexpr int ROW_PARTS = kCtaSums ? 1 : 64 / WTN;    // fused row sums of a BS = 64 block
 constexpr int A_BYTES = TILE * BK * 8;      // 8 KiB
 constexpr int B_BYTES = BK * TN * 8;        // 8 KiB (TN 64) / 4 KiB (TN 32)
 constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 constexpr int MAXF = 64;                    // faults per 64x64 tile kept in smem (one per 8x8 block)
 constexpr int BOOK = 128;                   // barriers, counters, cursor
+constexpr int SUMBUF = 4 * 64 * 8;           // BS = 64 epilogue exchange (kCtaSums)
 constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + BOOK +
-                           MAXF * (int)sizeof(aabft_fault);
+                           MAXF * (int)sizeof(aabft_fault) + SUMBUF;
 constexpr int GROUP_M = AABFT_F64_GROUP_M;
 constexpr int kMaxCtas = 1024;              // >= resident CTAs; sizes the split-K partial slots
 constexpr int ACC = MT * NT * 4;            // accumulators per thread
@@ -395,6 +400,8 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
   int *s_nf = reinterpret_cast<int *>(empty + STAGES);
   static_assert(16 * STAGES + 8 <= BOOK, "bookkeeping fits");
   aabft_fault *s_f = reinterpret_cast<aabft_fault *>(smem + STAGES * STAGE_BYTES + BOOK);
+  double *s_csum = reinterpret_cast<double *>(s_f + MAXF);  // [2][64] column parts (row halves)
+  double *s_rsum = s_csum + 128;                              // [2][64] row parts (column halves)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int g = lane >> 2, tig = lane & 3;
@@ -655,6 +662,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
       // part 0 in Rcol/Rrow, the others in the workspace) that aabft_check adds in part order.
       const int bs = args.bs;
       const int64_t nJ = args.N / bs;
+      const bool cta64 = kCtaSums && bs == 64;  // block == CTA tile: complete the sums here
       // column sums: per (nt, e) column, 8-row trees over g, then (h, mt) pairwise
 #pragma unroll
       for (int nt = 0; nt < NT; ++nt)
@@ -687,6 +695,8 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
               const int64_t I0 = rbase / 16;
               if (I0 * 16 < args.M) args.Rcol[I0 * args.N + col] = c16a;
               if ((I0 + 1) * 16 < args.M) args.Rcol[(I0 + 1) * args.N + col] = c16b;
+            } else if (cta64) {  // each 32-row half of the column into the exchange buffer
+              s_csum[wm * 64 + wn * 32 + nt * 8 + tig * 2 + e] = c32;
             } else {  // 32 or 64: one value per warp; part = which 32-row half of the block
               const int64_t I = rbase / bs;
               const int part = (int)((rbase % bs) / 32);
@@ -727,6 +737,8 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
                 const int64_t J = (cbase + q * 16) / 16;
                 if (J < nJ) args.Rrow[row * nJ + J] = r16[q];
               }
+            } else if (cta64) {  // each 32-column half of the row into the exchange buffer
+              s_rsum[wn * 64 + wm * 32 + mt * 16 + h * 8 + g] = rw;
             } else if (bs < WTN) {  // bs = 32 inside a 32-column warp tile (NT == 4)
               const int64_t J = cbase / 32;
               if (J < nJ) args.Rrow[row * nJ + J] = rw;
@@ -738,6 +750,15 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
             }
           }
         }
+      if (cta64) {
+        // complete the block's sums in part order (rows / columns 0..31 first, then 32..63)
+        mma_sync_bar();
+        const int64_t I = tl.m0 / 64, J = tl.n0 / 64;
+        const int t = threadIdx.x;  // 128 MMA threads: column t / 64 ... one value each
+        if (t < 64) args.Rcol[I * args.N + tl.n0 + t] = s_csum[t] + s_csum[64 + t];
+        else args.Rrow[(tl.m0 + (t - 64)) * nJ + J] = s_rsum[t - 64] + s_rsum[t];
+        mma_sync_bar();  // the exchange buffers are free for the next tile
+      }
     }
     double *out;
     int64_t ld, rows_valid, cols_valid;
@@ -850,6 +871,10 @@ size_t gemm_f64_ws_bytes(const aabft_config *cfg) {
 // the unprotected GEMM: split-K partial slots and flags only
 size_t gemm_f64_plain_ws_bytes() { return tpv_off() + 256; }
 int gemm_f64_fused_parts(int bs, int *row_parts) {
+  if (kCtaSums) {  // every block's sums are complete after the epilogue
+    *row_parts = 1;
+    return 1;
+  }
   *row_parts = bs > WTN ? bs / WTN : 1;
   return bs > 32 ? bs / 32 : 1;
 }
