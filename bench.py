@@ -64,6 +64,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--campaign", type=int, default=1, help="fault-injection runs (0 = skip)")
+    ap.add_argument("--no-traffic", action="store_true",
+                    help="skip the ncu DRAM-traffic probe of the dominant kernel")
     return ap.parse_args()
 
 
@@ -350,13 +352,9 @@ def main():
     aug_flops = 2.0 * K * (m_local * N + (m_local // bs) * N + m_local * (N // bs))
     peak = DMMA_PEAK_TFLOPS if wl["dtype"] == "f64" else FFMA_PEAK_TFLOPS
     achieved = aug_flops / (gemm_avg * 1e-3) / 1e12
-    traffic = None
-    prof = os.path.join(ROOT, "profiles", "gemm_traffic.json")
-    if os.path.exists(prof):
-        try:
-            traffic = json.load(open(prof)).get(args.workload)
-        except Exception:
-            traffic = None
+    traffic, traffic_src = None, "not measured (--no-traffic or N > 1)"
+    if rank == 0 and world == 1 and not args.no_traffic:
+        traffic, traffic_src = measure_traffic(wl, m_local, N, K, bs)
 
     # per-stage device times of one protected step, and Table I's comparators (NEXT-3)
     stages = stage_times(plan, A, B, stream, dev, args.steps)
@@ -428,6 +426,7 @@ def main():
                          "kernel": "gemm_f64_kernel (DMMA)" if wl["dtype"] == "f64" else "gemm_f32_kernel (FFMA)",
                          "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
                          "frac": achieved / peak, "traffic": traffic,
+                         "traffic_source": traffic_src,
                          "peak_source": "measured mma.sync f64 / FFMA issue ceiling, profiles/r01_step0_pipes.jsonl",
                          "algorithmic_flops_per_launch": aug_flops,
                          "avg_launch_ms": gemm_avg,
@@ -439,6 +438,38 @@ def main():
         print(json.dumps(out), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def measure_traffic(wl, m_local, N, K, bs):
+    """roofline.traffic measured in this run: ncu (dram__bytes_read.sum + dram__bytes_write.sum)
+    on one launch of the dominant kernel of the same workload, in a subprocess after the timed
+    region (tools/traffic_probe.py; its own process, so the bench's timings are unaffected).
+    Returns (bytes per launch, source) or (None, reason)."""
+    import shutil
+    ncu = shutil.which("ncu") or "/usr/local/cuda/bin/ncu"
+    if not os.path.exists(ncu):
+        return None, "ncu not found"
+    kern = "gemm_f64_kernel" if wl["dtype"] == "f64" else "gemm_f32_kernel"
+    cmd = [ncu, "--metrics", "dram__bytes_read.sum,dram__bytes_write.sum", "--clock-control",
+           "none", "-k", "regex:" + kern, "-s", "1", "-c", "1", "--csv", sys.executable,
+           os.path.join(ROOT, "tools", "traffic_probe.py"), str(m_local), str(N), str(K), str(bs),
+           wl["dtype"], wl["recipe"]]
+    try:
+        r = subprocess.run(cmd, capture_output=True, text=True, timeout=240)
+    except Exception as e:  # timeout / missing permissions: report, do not fail the bench
+        return None, f"ncu probe failed: {e!r}"[:200]
+    import csv
+    total = 0.0
+    seen = 0
+    for row in csv.reader(l for l in r.stdout.splitlines() if l.startswith('"')):
+        if len(row) > 14 and row[12] in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
+            unit, val = row[13], float(row[14].replace(",", ""))
+            scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}.get(unit, 1)
+            total += val * scale
+            seen += 1
+    if seen != 2:
+        return None, "ncu probe: metrics not found (" + (r.stderr or r.stdout)[-160:] + ")"
+    return total, f"ncu dram__bytes_read+write.sum, one {kern} launch, same shape, this run"
 
 
 def stage_times(plan, A, B, stream, dev, steps):
