@@ -38,6 +38,9 @@ namespace {
 #ifndef AABFT_F64_STAGES
 #define AABFT_F64_STAGES 4
 #endif
+#ifndef AABFT_F64_PROD_FIRST
+#define AABFT_F64_PROD_FIRST 0
+#endif
 #ifndef AABFT_F64_B3D
 #define AABFT_F64_B3D 0
 #endif
@@ -403,7 +406,12 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
   double *s_csum = reinterpret_cast<double *>(s_f + MAXF);  // [2][64] column parts (row halves)
   double *s_rsum = s_csum + 128;                              // [2][64] row parts (column halves)
 
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  // warp roles: the producer is the CTA's last warp (AABFT_F64_PROD_FIRST: its first);
+  // mtid / mwarp index the 4 MMA warps
+  const int warp_hw = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int prod_warp = AABFT_F64_PROD_FIRST ? 0 : NCW;
+  const int warp = AABFT_F64_PROD_FIRST ? (warp_hw == 0 ? NCW : warp_hw - 1) : warp_hw;
+  const int mtid = warp * 32 + lane;  // MMA thread index 0..THREADS-1 (producer: THREADS..)
   const int g = lane >> 2, tig = lane & 3;
   const int wm = warp / WARPS_N, wn = warp % WARPS_N;
 
@@ -423,7 +431,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
   // ---------------- TMA producer warp: streams every job of this CTA through the ring,
   // refilling a stage as soon as the 4 MMA warps released it (empty mbarrier).  The box
   // copies are spread over the lanes (one cp.async.bulk.tensor per lane).
-  if (warp == NCW) {
+  if (warp_hw == prod_warp) {
     if (lane == 0) {
       tma_prefetch_desc(&tmA);
       tma_prefetch_desc(&tmB);
@@ -498,9 +506,9 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
     int nf = 0;
     if (FAULTS && args.nfaults > 0) {
       mma_sync_bar();
-      if (threadIdx.x == 0) *s_nf = 0;
+      if (mtid == 0) *s_nf = 0;
       mma_sync_bar();
-      for (int f = threadIdx.x; f < args.nfaults; f += THREADS) {
+      for (int f = mtid; f < args.nfaults; f += THREADS) {
         aabft_fault ft = args.faults[f];
         int64_t r = ft.row, c = ft.col;
         int ftype;
@@ -602,7 +610,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
     const bool first = kt0 == 0, last = kt_end == args.nk;
     if (!first) {
       // contributor: park the partial accumulators, then signal the owner
-      double *slot = args.partials + (int64_t)blockIdx.x * ACC * THREADS + threadIdx.x;
+      double *slot = args.partials + (int64_t)blockIdx.x * ACC * THREADS + mtid;
 #pragma unroll
       for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
@@ -611,7 +619,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
           for (int q = 0; q < 4; ++q) slot[((mt * NT + nt) * 4 + q) * THREADS] = acc[mt][nt][q];
       __threadfence();
       mma_sync_bar();
-      if (threadIdx.x == 0) atomicExch(&args.flags[blockIdx.x], 1);
+      if (mtid == 0) atomicExch(&args.flags[blockIdx.x], 1);
       continue;
     }
     if (!last) {
@@ -619,13 +627,13 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
       const int64_t tile_it_end = (int64_t)(tile - args.waves * (int)gridDim.x + 1) * args.nk;
       for (int64_t c = blockIdx.x + 1; c < gridDim.x && sk_begin(args, c) < tile_it_end; ++c) {
         if (sk_begin(args, c + 1) == sk_begin(args, c)) continue;  // empty slice: no partial
-        if (threadIdx.x == 0) {
+        if (mtid == 0) {
           while (atomicAdd(&args.flags[c], 0) == 0) __nanosleep(64);
           atomicExch(&args.flags[c], 0);  // re-arm for the next launch
           __threadfence();
         }
         mma_sync_bar();
-        const double *slot = args.partials + c * ACC * THREADS + threadIdx.x;
+        const double *slot = args.partials + c * ACC * THREADS + mtid;
 #pragma unroll
         for (int mt = 0; mt < MT; ++mt)
 #pragma unroll
@@ -754,7 +762,7 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
         // complete the block's sums in part order (rows / columns 0..31 first, then 32..63)
         mma_sync_bar();
         const int64_t I = tl.m0 / 64, J = tl.n0 / 64;
-        const int t = threadIdx.x;  // 128 MMA threads: column t / 64 ... one value each
+        const int t = mtid;  // 128 MMA threads: column t / 64 ... one value each
         if (t < 64) args.Rcol[I * args.N + tl.n0 + t] = s_csum[t] + s_csum[64 + t];
         else args.Rrow[(tl.m0 + (t - 64)) * nJ + J] = s_rsum[t - 64] + s_rsum[t];
         mma_sync_bar();  // the exchange buffers are free for the next tile
