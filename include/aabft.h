@@ -83,6 +83,12 @@ typedef struct {
  * contents (value desc, index asc; bit-exact).  Opt-in: on B200 it measured slower than the
  * selection in aabft_encode. */
 #define AABFT_FLAG_TOPP_IN_GEMM 1
+/* AABFT_FLAG_GEMM_HALF_GRID: the FP64 aabft_gemm / aabft_gemm_plain launch uses half of the
+ * persistent grid (1.5 CTAs per SM) so that two such calls on two streams can run side by side
+ * (the host entry point's pipelined blocks use it).  A launch with a stream-K tail is
+ * cooperative, so each grid is fully resident before it starts.  Results are identical up to
+ * the FP64 summation order of split tiles (parity by tolerance, as always for FP64). */
+#define AABFT_FLAG_GEMM_HALF_GRID 2
 
 /* Output of aabft_encode.  Acs: (M/bs) x K, ld_acs >= K.  Bcs: K x (N/bs), ld_bcs >= N/bs.
  * topA_val/topA_idx: (M + M/bs) x p -- data rows 0..M-1, then checksum rows; |value|

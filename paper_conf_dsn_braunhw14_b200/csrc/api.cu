@@ -423,7 +423,7 @@ int64_t piece(int64_t total, int64_t step, int i) {
 struct Arena {
   int64_t lda, ldb, ldc, ld_acs, ld_bcs, ld_ccol, ld_crow;
   size_t oA, oB, oC, oAcs, oBcs, oCcol, oCrow, oRcol, oRrow, oTav, oTai, oTbv, oTbi, oRep, oCnt,
-      oCntAll, oWs, total;
+      oCntAll, oWs, oWs2, total;
 };
 Arena plan_arena(const aabft_config *c) {
   Arena a;
@@ -453,12 +453,14 @@ Arena plan_arena(const aabft_config *c) {
   a.oCnt = take(sizeof(aabft_counts) * sp.S * sp.S);
   a.oCntAll = take(sizeof(aabft_counts));
   a.oWs = take(aabft_workspace_bytes(c));
+  a.oWs2 = take(aabft_workspace_bytes(c));  // the second compute stream's workspace
   a.total = o;
   return a;
 }
-struct HostPipe {  // per-device copy streams + event pool (created once; the library's runtime)
-  cudaStream_t in = nullptr, out = nullptr;
+struct HostPipe {  // per-device copy / compute streams + event pool (created once)
+  cudaStream_t in = nullptr, out = nullptr, c2 = nullptr;
   cudaEvent_t ev[2 * kMaxSplit + kMaxSplit * kMaxSplit + 2];
+  cudaEvent_t enc[2 * kMaxSplit + 2];  // encode of A_i / B_j done; second stream done
   bool ok = false;
 };
 HostPipe &host_pipe() {
@@ -468,9 +470,12 @@ HostPipe &host_pipe() {
   HostPipe &h = hp[dev & 63];
   if (!h.ok) {
     if (cudaStreamCreateWithFlags(&h.in, cudaStreamNonBlocking) != cudaSuccess ||
-        cudaStreamCreateWithFlags(&h.out, cudaStreamNonBlocking) != cudaSuccess)
+        cudaStreamCreateWithFlags(&h.out, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaStreamCreateWithFlags(&h.c2, cudaStreamNonBlocking) != cudaSuccess)
       return h;
     for (auto &e : h.ev)
+      if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return h;
+    for (auto &e : h.enc)
       if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return h;
     h.ok = true;
   }
@@ -509,8 +514,15 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
   cudaEvent_t evOutDone = hp.ev[2 * kMaxSplit + kMaxSplit * kMaxSplit + 1];
   // the copy streams start after whatever the caller enqueued before this call
   if (cudaEventRecord(evStart, st) != cudaSuccess || cudaStreamWaitEvent(hp.in, evStart, 0) != cudaSuccess ||
-      cudaStreamWaitEvent(hp.out, evStart, 0) != cudaSuccess)
+      cudaStreamWaitEvent(hp.out, evStart, 0) != cudaSuccess ||
+      cudaStreamWaitEvent(hp.c2, evStart, 0) != cudaSuccess)
     return check_launch("pipeline start");
+  // two compute streams: consecutive blocks alternate between them and each FP64 GEMM runs on
+  // half the persistent grid (AABFT_FLAG_GEMM_HALF_GRID), so one block's stream-K tail
+  // overlaps the next block's data-parallel waves instead of idling SMs
+  const bool two = cfg->dtype == AABFT_F64 && sp.S > 1 && !std::getenv("AABFT_HOST_ONE_STREAM");
+  cudaEvent_t *evEncA = hp.enc, *evEncB = hp.enc + kMaxSplit;
+  cudaEvent_t evC2Done = hp.enc[2 * kMaxSplit];
   // AABFT_HOST_TRACE=1: timing events per copy / block, printed to stderr after the call
   // (diagnostics for the pipeline's schedule; no effect on results)
   static const bool trace = std::getenv("AABFT_HOST_TRACE") != nullptr;
@@ -573,20 +585,32 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
       aabft_config cb = *cfg;
       cb.M = mi;
       cb.N = nj;
+      if (two) cb.flags |= AABFT_FLAG_GEMM_HALF_GRID;
+      const bool second = two && (nblk & 1);
+      cudaStream_t cs = second ? hp.c2 : st;
+      void *ws = base + (second ? a.oWs2 : a.oWs);
       const void *Ai = base + a.oA + (size_t)(i * sp.ms) * a.lda * es;
       const void *Bj = base + a.oB + (size_t)(j * sp.ns) * es;
       aabft_encoded enc{base + a.oAcs + (size_t)(i * sp.ms / bs) * a.ld_acs * es, a.ld_acs,
                         base + a.oBcs + (size_t)(j * sp.ns / bs) * es, a.ld_bcs,
                         tav(i), tai(i), tbv(j), tbi(j)};
+      // encode a newly arrived slab / panel once (on this block's stream); blocks on the other
+      // stream wait for that encode's event
       if (!encA[i]) {
-        cudaStreamWaitEvent(st, evA[i], 0);
-        if ((s = aabft_encode(&cb, Ai, a.lda, nullptr, 0, &enc, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
+        cudaStreamWaitEvent(cs, evA[i], 0);
+        if ((s = aabft_encode(&cb, Ai, a.lda, nullptr, 0, &enc, ws, wsb, cs)) != AABFT_OK) return s;
+        cudaEventRecord(evEncA[i], cs);
         encA[i] = true;
+      } else {
+        cudaStreamWaitEvent(cs, evEncA[i], 0);
       }
       if (!encB[j]) {
-        cudaStreamWaitEvent(st, evB[j], 0);
-        if ((s = aabft_encode(&cb, nullptr, 0, Bj, a.ldb, &enc, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
+        cudaStreamWaitEvent(cs, evB[j], 0);
+        if ((s = aabft_encode(&cb, nullptr, 0, Bj, a.ldb, &enc, ws, wsb, cs)) != AABFT_OK) return s;
+        cudaEventRecord(evEncB[j], cs);
         encB[j] = true;
+      } else {
+        cudaStreamWaitEvent(cs, evEncB[j], 0);
       }
       aabft_product prod{base + a.oC + ((size_t)(i * sp.ms) * a.ldc + (size_t)(j * sp.ns)) * es, a.ldc,
                          base + a.oCcol + ((size_t)(i * sp.ms / bs) * a.ld_ccol + (size_t)(j * sp.ns)) * es, a.ld_ccol,
@@ -598,12 +622,12 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
       rrow_off += r256((size_t)mi * (nj / bs) * 8);
       rep_off += r256((size_t)(mi / bs) * (nj / bs) * sizeof(aabft_block_report));
       aabft_counts *cnt = cnt_blocks + nblk;
-      if ((s = aabft_gemm(&cb, Ai, a.lda, Bj, a.ldb, &enc, &prod, nullptr, 0, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
-      if ((s = aabft_check(&cb, &enc, &prod, rep, cnt, base + a.oWs, wsb, stream)) != AABFT_OK) return s;
-      if ((s = aabft_correct(&cb, &enc, &prod, rep, cnt, stream)) != AABFT_OK) return s;
+      if ((s = aabft_gemm(&cb, Ai, a.lda, Bj, a.ldb, &enc, &prod, nullptr, 0, ws, wsb, cs)) != AABFT_OK) return s;
+      if ((s = aabft_check(&cb, &enc, &prod, rep, cnt, ws, wsb, cs)) != AABFT_OK) return s;
+      if ((s = aabft_correct(&cb, &enc, &prod, rep, cnt, cs)) != AABFT_OK) return s;
       // device -> host of the finished (corrected) C block on the copy-out stream
-      cudaEventRecord(evC[nblk], st);
-      mark(st, "block done", i, j);
+      cudaEventRecord(evC[nblk], cs);
+      mark(cs, "block done", i, j);
       cudaStreamWaitEvent(hp.out, evC[nblk], 0);
       if (cudaMemcpy2DAsync(static_cast<char *>(C_host) + ((size_t)(i * sp.ms) * N + (size_t)(j * sp.ns)) * es,
                             N * es, prod.C, a.ldc * es, nj * es, mi, cudaMemcpyDeviceToHost, hp.out) != cudaSuccess)
@@ -622,7 +646,11 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
       if ((s = ord_kind[o] == 0 ? run_block(x, y) : run_block(y, x)) != AABFT_OK) return s;
     }
   }
-  // global counters = sum over the blocks (SUM n, MAX max_ratio)
+  // global counters = sum over the blocks (SUM n, MAX max_ratio), after both compute streams
+  if (two) {
+    cudaEventRecord(evC2Done, hp.c2);
+    cudaStreamWaitEvent(st, evC2Done, 0);
+  }
   auto *cnt_all = reinterpret_cast<aabft_counts *>(base + a.oCntAll);
   if ((s = launch_counts_sum(cnt_blocks, nblk, cnt_all, st)) != AABFT_OK) return s;
   if (counts_host && cudaMemcpyAsync(counts_host, cnt_all, sizeof(aabft_counts), cudaMemcpyDeviceToHost, st) != cudaSuccess)

@@ -417,7 +417,10 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
 
   // this CTA's k-tile sequence: its data-parallel tiles, then its stream-K slice
   const int64_t sk0 = sk_begin(args, blockIdx.x), sk1 = sk_begin(args, blockIdx.x + 1);
-  const int njobs = args.waves * args.nk + (int)(sk1 - sk0);
+  // data-parallel tiles of this CTA (the last wave may be partial when there is no stream-K
+  // tail: AABFT_FLAG_GEMM_HALF_GRID), then its stream-K slice
+  const int my_dp = min(args.waves, ((int)args.ntiles - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x);
+  const int njobs = my_dp * args.nk + (int)(sk1 - sk0);
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < STAGES; ++s) {
@@ -946,13 +949,15 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
   a.ntiles = (int)ntiles;
   a.nk = (int)nk;
   const int64_t total = ntiles * nk;
-  const int grid = (int)std::min<int64_t>(max_ctas, total);
+  // AABFT_FLAG_GEMM_HALF_GRID: half the persistent grid, so two launches can share the GPU
+  const int cap = (cfg->flags & AABFT_FLAG_GEMM_HALF_GRID) ? std::max(1, max_ctas / 2) : max_ctas;
+  const int grid = (int)std::min<int64_t>(cap, total);
   // full data-parallel waves, keeping at least ~1/2 wave of tiles for the stream-K tail so
   // every CTA's k-slice stays long enough to amortise its fixup
   int waves = (int)(ntiles / grid);
   if (waves > 0 && ntiles % grid != 0 && (ntiles % grid) * 2 < grid) waves -= 1;
   a.waves = waves;
-  a.sk_iters = (ntiles - (int64_t)waves * grid) * nk;
+  a.sk_iters = std::max<int64_t>(0, ntiles - (int64_t)waves * grid) * nk;
   a.partials = static_cast<double *>(ws);
   a.flags = reinterpret_cast<int *>(static_cast<char *>(ws) + flags_off());
   a.tp_flags = a.flags + kMaxCtas;

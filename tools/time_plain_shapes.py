@@ -12,7 +12,10 @@ def t(fn, reps=10):
         e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
         e0.record(); fn(); e1.record(); torch.cuda.synchronize(); ts.append(e0.elapsed_time(e1))
     return float(np.median(ts))
-for M, N, K in [(4096, 4096, 4096), (9472, 3072, 4096), (9472, 3072, 1024), (9472, 6144, 4096), (4736, 3072, 8192)]:
+SHAPES = [(4096, 4096, 4096), (9472, 3072, 4096), (9472, 3072, 1024), (9472, 6144, 4096), (4736, 3072, 8192)]
+if len(sys.argv) > 1:
+    SHAPES = [tuple(int(x) for x in a.split('x')) for a in sys.argv[1:]]
+for M, N, K in SHAPES:
     A = torch.rand(M, K, dtype=torch.float64, device="cuda"); B = torch.rand(K, N, dtype=torch.float64, device="cuda")
     C = torch.empty(M, N, dtype=torch.float64, device="cuda")
     ms = t(lambda: api.gemm_plain(A, B, out=C))
