@@ -110,11 +110,11 @@ typedef struct {
  * checksums c_{i,q+1} per block-column (Eq 3 with partitioned encoding; corner not formed,
  * reading R17).
  * Rcol / Rrow (optional, double, dense (M/bs) x N and M x (N/bs)): when both are non-NULL and
- * the FP64 path runs with bs <= 64, aabft_gemm also forms the REFERENCE checksums of Eq 4
- * (c*_{m+1,j}, c*_{i,q+1}) from its epilogue registers (for bs = 64 as two partial halves,
- * the second one in the workspace) and aabft_check -- which then needs the same workspace --
- * compares those instead of re-reading C ("fused check"); after aabft_check Rcol / Rrow
- * hold the complete reference sums.  NULL = unfused: aabft_check re-sums C. */
+ * the path supports it (FP64 with bs <= 64, FP32 with bs <= 128), aabft_gemm also forms the
+ * REFERENCE checksums of Eq 4 (c*_{m+1,j}, c*_{i,q+1}) from its epilogue registers and
+ * aabft_check -- which then needs the same workspace -- compares those instead of re-reading C
+ * ("fused check"; fault model: DESIGN.md 6.4); after aabft_check Rcol / Rrow hold the
+ * complete reference sums.  NULL = unfused: aabft_check re-sums C. */
 typedef struct {
   void *C;
   int64_t ldc;

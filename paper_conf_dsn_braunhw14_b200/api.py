@@ -157,8 +157,9 @@ class ProtectedGemm:
         self.enc_cs = Encoded(self._Acs.data_ptr(), self.ld_acs, self._Bcs.data_ptr(),
                               self.ld_bcs, None, None, None, None)
         self._sea = None
-        # fused check (FP64, bs <= 64): the GEMM epilogue writes the reference sums
-        self.fused = bool(fused and dtype == torch.float64 and bs <= 64)
+        # fused check (FP64 bs <= 64, FP32 bs <= 128): the GEMM epilogue writes the reference sums
+        self.fused = bool(fused and ((dtype == torch.float64 and bs <= 64) or
+                                     (dtype == torch.float32 and bs <= 128)))
         self.Rcol = torch.empty(nI, N, dtype=torch.float64, device=dev) if self.fused else None
         self.Rrow = torch.empty(M, nJ, dtype=torch.float64, device=dev) if self.fused else None
         self.prod = Product(self._C.data_ptr(), self.ldc, self._Ccol.data_ptr(), self.ld_ccol,

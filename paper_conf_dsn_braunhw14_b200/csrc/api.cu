@@ -298,7 +298,7 @@ aabft_status aabft_check(const aabft_config *cfg, const aabft_encoded *enc,
   AABFT_GUARD_BEGIN
   aabft_status s = check_common(cfg, enc, prod, reports, counts);
   if (s != AABFT_OK) return s;
-  const bool fused = prod->Rcol && prod->Rrow && cfg->dtype == AABFT_F64 && cfg->bs <= 64;
+  const bool fused = prod->Rcol && prod->Rrow && fused_check_ok(cfg);
   if (fused && (!ws || ws_bytes < aabft_workspace_bytes(cfg))) {
     set_error("check (fused): the aabft_gemm workspace is required");
     return AABFT_EWORKSPACE;
@@ -363,7 +363,7 @@ aabft_status aabft_check_ext(const aabft_config *cfg, const aabft_product *prod,
   AABFT_GUARD_BEGIN
   aabft_status s = ext_common(cfg, prod, eps_fixed, reports, counts);
   if (s != AABFT_OK) return s;
-  const bool fused = prod->Rcol && prod->Rrow && cfg->dtype == AABFT_F64 && cfg->bs <= 64;
+  const bool fused = prod->Rcol && prod->Rrow && fused_check_ok(cfg);
   if (fused && (!ws || ws_bytes < aabft_workspace_bytes(cfg))) {
     set_error("check_ext (fused): the aabft_gemm workspace is required");
     return AABFT_EWORKSPACE;

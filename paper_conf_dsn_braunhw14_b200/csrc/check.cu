@@ -560,14 +560,14 @@ CheckArgs make_args(const aabft_config *cfg, const aabft_encoded *enc, const aab
   a.tbv = enc ? enc->topB_val : nullptr; a.tbi = enc ? enc->topB_idx : nullptr;
   a.rep = rep; a.cnt = cnt;
   // fused reference sums exist only where aabft_gemm produces them (FP64, bs <= 64)
-  const bool fused = prod->Rcol && prod->Rrow && cfg->dtype == AABFT_F64 && cfg->bs <= 64;
+  const bool fused = prod->Rcol && prod->Rrow && fused_check_ok(cfg);
   a.Rcol = fused && gemm_ws ? prod->Rcol : nullptr;
   a.Rrow = fused && gemm_ws ? prod->Rrow : nullptr;
   a.Rcol2 = a.Rrow2 = nullptr;
   a.col_parts = a.row_parts = 1;
   a.eps_col = a.eps_row = nullptr;
   a.eps_fixed = 0.0;
-  if (a.Rcol) {
+  if (a.Rcol && cfg->dtype == AABFT_F64) {  // the FP32 epilogue always completes its sums
     a.col_parts = gemm_f64_fused_parts(cfg->bs, &a.row_parts);
     double *rc2, *rr2;
     gemm_f64_red_ptrs(cfg, gemm_ws, &rc2, &rr2);
@@ -580,7 +580,7 @@ CheckArgs make_args(const aabft_config *cfg, const aabft_encoded *enc, const aab
 // correction: the fused reference sums (complete after aabft_check) are refreshed for every
 // corrected element (a second check of a corrected product must stay clean)
 void set_refresh(const aabft_config *cfg, const aabft_product *prod, CheckArgs &a) {
-  const bool fused = prod->Rcol && prod->Rrow && cfg->dtype == AABFT_F64 && cfg->bs <= 64;
+  const bool fused = prod->Rcol && prod->Rrow && fused_check_ok(cfg);
   a.Rcol = fused ? prod->Rcol : nullptr;
   a.Rrow = fused ? prod->Rrow : nullptr;
 }

@@ -17,6 +17,12 @@ aabft_status validate(const aabft_config *cfg);
 int eff_t(const aabft_config *cfg);
 size_t elem_size(const aabft_config *cfg);
 
+// the GEMM epilogue forms the reference sums of the check (fused check): FP64 with bs <= 64
+// (64 x 64 tiles), FP32 with bs <= 128 (128 x 128 tiles)
+inline bool fused_check_ok(const aabft_config *cfg) {
+  return (cfg->dtype == AABFT_F64 && cfg->bs <= 64) || (cfg->dtype == AABFT_F32 && cfg->bs <= 128);
+}
+
 // sigma coefficient sqrt(F(K)) (Eq 28 P:L219 / P:L287) evaluated in double on the host
 // (compiled without FMA contraction); passed to kernels as a parameter.
 double sigma_coeff(int64_t K, int fma_model);

@@ -34,7 +34,9 @@ constexpr int BM = 128, BN = AABFT_F32_BN, BK = AABFT_F32_BK, STAGES = AABFT_F32
 constexpr int TX = BN / 8, THREADS = 16 * TX;   // 16 x TX threads, 8 x 8 outputs each
 constexpr int HN = BN / 2;                      // column offset of the second 4-wide half
 constexpr int MAXF = BM * BN / 64;  // faults per tile kept in smem (one per 8x8 block)
-constexpr int SMEM32 = STAGES * (BM + BN) * BK * 4 + MAXF * (int)sizeof(aabft_fault);
+constexpr int RING32 = STAGES * (BM + BN) * BK * 4;
+constexpr int TILE32 = BM * (BN + 1) * 4;  // fused-sum epilogue staging (reuses the ring)
+constexpr int SMEM32 = (RING32 > TILE32 ? RING32 : TILE32) + MAXF * (int)sizeof(aabft_fault);
 #ifndef AABFT_F32_GROUP_M
 #define AABFT_F32_GROUP_M 8
 #endif
@@ -60,6 +62,9 @@ struct SgemmArgs {
   int tm0, tn0, tm1, tn2;
   const aabft_fault *faults;
   int nfaults;
+  double *Rcol;  // fused reference sums (NULL = unfused): (M/bs) x N, M x (N/bs)
+  double *Rrow;
+  int bs;
 };
 
 __device__ __forceinline__ float xor_bits(float v, uint64_t m) {
@@ -88,7 +93,7 @@ __global__ void __launch_bounds__(THREADS, AABFT_F32_MINB) gemm_f32_kernel(const
   extern __shared__ __align__(16) uint8_t smem32[];
   auto As = reinterpret_cast<float(*)[BM][BK]>(smem32);                          // [STAGES]
   auto Bs = reinterpret_cast<float(*)[BK][BN]>(smem32 + STAGES * BM * BK * 4);   // [STAGES]
-  aabft_fault *s_f = reinterpret_cast<aabft_fault *>(smem32 + STAGES * (BM + BN) * BK * 4);
+  aabft_fault *s_f = reinterpret_cast<aabft_fault *>(smem32 + (RING32 > TILE32 ? RING32 : TILE32));
   __shared__ int s_nf;
 
   int64_t bid = blockIdx.x;
@@ -272,6 +277,46 @@ __global__ void __launch_bounds__(THREADS, AABFT_F32_MINB) gemm_f32_kernel(const
         }
     }
   }
+  if (type == 0 && args.Rcol != nullptr) {
+    // ---- fused reference sums (Eq 4, in double, reading R12) of the BS x BS blocks of this
+    // 128 x 128 tile, from the registers about to be stored (after any injected fault): the
+    // check compares them instead of re-reading C (the FP64 kernel's design).  The tile goes
+    // through shared memory (the drained cp.async ring; odd pitch 129: conflict-free column AND
+    // row walks), then thread c < 128 sums column c down each block and thread 128 + r sums
+    // row r across each block, both in ascending order -- the definition's sequential order,
+    // so these sums equal the unfused check's bit for bit.
+    const int bs = args.bs;
+    __syncthreads();  // every warp is done with the stage buffers
+    float *s_tile = reinterpret_cast<float *>(smem32);  // [BM][BN + 1]
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const int r = i < 4 ? ty * 4 + i : 64 + ty * 4 + i - 4;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const int c = j < 4 ? tx * 4 + j : HN + tx * 4 + (j - 4);
+        s_tile[r * (BN + 1) + c] = ACC(i, j);
+      }
+    }
+    __syncthreads();
+    if (tid < BN) {  // column sums: rows of each block in ascending order
+      const int c = tid;
+      const int64_t col = n0 + c;
+      for (int r0 = 0; r0 < BM; r0 += bs) {
+        double sum = 0.0;
+        for (int r = r0; r < r0 + bs; ++r) sum = sum + (double)s_tile[r * (BN + 1) + c];
+        if (m0 + r0 < args.M && col < args.N) args.Rcol[((m0 + r0) / bs) * args.N + col] = sum;
+      }
+    } else if (tid < BN + BM) {  // row sums: columns of each block in ascending order
+      const int r = tid - BN;
+      const int64_t row = m0 + r, nJ = args.N / bs;
+      for (int c0 = 0; c0 < BN; c0 += bs) {
+        double sum = 0.0;
+        for (int c = c0; c < c0 + bs; ++c) sum = sum + (double)s_tile[r * (BN + 1) + c];
+        const int64_t J = (n0 + c0) / bs;
+        if (row < args.M && J < nJ) args.Rrow[row * nJ + J] = sum;
+      }
+    }
+  }
   float *out;
   int64_t ld;
   if (type == 0) { out = args.C; ld = args.ldc; }
@@ -330,6 +375,10 @@ aabft_status launch_gemm_f32(const aabft_config *cfg, const void *A, int64_t lda
   a.n2 = (int64_t)a.tm0 * a.tn2;
   a.faults = faults;
   a.nfaults = faults ? nfaults : 0;
+  a.bs = (int)bs;
+  const bool fused = !plain && out->Rcol && out->Rrow && fused_check_ok(cfg);
+  a.Rcol = fused ? out->Rcol : nullptr;
+  a.Rrow = fused ? out->Rrow : nullptr;
   const int64_t tiles = a.n0 + a.n1 + a.n2;
   static std::atomic<bool> attr_dev[64];  // per device (function attributes are per context)
   int dev = 0;

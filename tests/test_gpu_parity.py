@@ -371,6 +371,8 @@ def _fault_set(orc, A, B, bs, p, rng, dtype, n_per_mag=1):
 @pytest.mark.parametrize("dtype,fused,bs", [(np.float64, True, 64), (np.float64, False, 64),
                                             (np.float64, True, 32), (np.float64, True, 16),
                                             (np.float64, True, 8), (np.float32, False, 64),
+                                            (np.float32, True, 64), (np.float32, True, 8),
+                                            (np.float32, True, 128),
                                             # unfused streaming check: many / one / wide blocks
                                             (np.float32, False, 8), (np.float32, False, 128),
                                             (np.float64, False, 128), (np.float64, False, 256)])
@@ -381,7 +383,7 @@ def test_fault_verdicts_outside_band(P, orc, dtype, fused, bs):
     B = gen("uniform", K, N, 11, 1, dtype)
     faults, labels = _fault_set(orc, A, B, bs, p, rng, dtype)
     plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=p, fused=fused)
-    assert plan.fused == (fused and dtype == np.float64)
+    assert plan.fused == (fused and (bs <= 64 if dtype == np.float64 else bs <= 128))
     dA, dB = to_dev(A), to_dev(B)
     clean = host(plan.run(dA, dB).C).copy()
     res = plan.run(dA, dB, faults=faults)
@@ -618,17 +620,20 @@ def test_distributed_single_rank_nccl(P, orc):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("bs", [8, 16, 32, 64])
-def test_fused_reference_sums(P, orc, bs):
-    """The epilogue reference sums (completed by aabft_check) equal the definition (Eq 4) up to
-    summation order."""
-    M, N, K = 320, 192, 300
-    A = gen("uniform", M, K, 31, 0)
-    B = gen("uniform", K, N, 31, 1)
-    plan = P.ProtectedGemm(M, N, K, dtype=torch.float64, bs=bs, p=2)
+@pytest.mark.parametrize("dtype,bs", [(np.float64, 8), (np.float64, 16), (np.float64, 32),
+                                      (np.float64, 64), (np.float32, 8), (np.float32, 16),
+                                      (np.float32, 32), (np.float32, 64), (np.float32, 128)])
+def test_fused_reference_sums(P, orc, dtype, bs):
+    """The epilogue reference sums (complete after aabft_check) equal the definition (Eq 4) up to
+    summation order -- FP64 (64 x 64 DMMA tiles) and FP32 (128 x 128 FFMA tiles)."""
+    M, N, K = 384, 256, 300
+    A = gen("uniform", M, K, 31, 0, dtype)
+    B = gen("uniform", K, N, 31, 1, dtype)
+    plan = P.ProtectedGemm(M, N, K, dtype=TD[dtype], bs=bs, p=2)
+    assert plan.fused
     res = plan.run(to_dev(A), to_dev(B))
     torch.cuda.synchronize()
-    C = host(res.C)
+    C = host(res.C).astype(np.float64)
     Rcol = C.reshape(M // bs, bs, N).sum(axis=1)
     Rrow = C.reshape(M, N // bs, bs).sum(axis=2)
     scale = np.abs(C).max() * bs
