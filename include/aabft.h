@@ -89,6 +89,21 @@ typedef struct {
  * cooperative, so each grid is fully resident before it starts.  Results are identical up to
  * the FP64 summation order of split tiles (parity by tolerance, as always for FP64). */
 #define AABFT_FLAG_GEMM_HALF_GRID 2
+/* AABFT_FLAG_OVERLAP_ENCODE: step 1 runs CONCURRENTLY with the following aabft_gemm on the same
+ * stream (the paper overlaps its top-p reduction with the multiplication, P:L320 / P:L368;
+ * here the whole encode does).  aabft_encode (FP64, 16 <= bs <= 64, p <= 4, A, B and both
+ * top-p tables given; otherwise the flag is ignored) launches a one-CTA-per-SM kernel small
+ * enough to sit next to the GEMM's CTAs and marks the GEMM as a programmatic dependent launch;
+ * aabft_gemm (FP64) then streams its data tiles at once and waits for the encode grid only
+ * before its first checksum tile.  Results are bit-identical to the unflagged calls.  Pass
+ * the flag to BOTH calls (and to aabft_check / aabft_correct, which ignore it).  Contract:
+ * the workspace must be zero-filled once before its first flagged aabft_gemm (the kernel
+ * leaves its split-K flag words zero after every launch, so no per-call reset -- which would
+ * sit between the two kernels and serialise them -- is needed).  Opt-in: measured SLOWER on
+ * B200 -- the encode's FP64 additions share the FP64 datapath with the GEMM's
+ * DMMA instructions, which stretches the co-resident encode 7x and costs the GEMM more than
+ * the serial encode takes. */
+#define AABFT_FLAG_OVERLAP_ENCODE 4
 
 /* Output of aabft_encode.  Acs: (M/bs) x K, ld_acs >= K.  Bcs: K x (N/bs), ld_bcs >= N/bs.
  * topA_val/topA_idx: (M + M/bs) x p -- data rows 0..M-1, then checksum rows; |value|

@@ -113,12 +113,19 @@ class ProtectedGemm:
 
     def __init__(self, M: int, N: int, K: int, *, dtype=torch.float64, bs: int = 64, p: int = 2,
                  omega: float = 3.0, t: int = 0, fma_model: int = 1, device=None,
-                 fused: bool = True, topp_in_gemm: bool = False):
+                 fused: bool = True, topp_in_gemm: bool = False, overlap: bool = False):
         lib()  # fail loudly before allocating anything
         self.device = torch.device("cuda" if device is None else device)
         self.dtype = dtype
         self.M, self.N, self.K, self.bs, self.p = M, N, K, bs, p
-        self.cfg = Config(_dtype_code(dtype), bs, M, N, K, p, t, omega, fma_model, 0)
+        # AABFT_FLAG_OVERLAP_ENCODE (include/aabft.h): the encode runs concurrently with the
+        # GEMM's data tiles (FP64, 16 <= bs <= 64, p <= 4; ignored elsewhere).  Bit-identical
+        # results; the workspace is zero-filled once below, as the flag's contract requires.
+        # Opt-in: measured slower on B200 (the encode's FP64 adds stall the GEMM's DMMA pipe,
+        # DESIGN.md 8.11).
+        self.overlap = bool(overlap and dtype == torch.float64 and 16 <= bs <= 64 and p <= 4)
+        self.cfg = Config(_dtype_code(dtype), bs, M, N, K, p, t, omega, fma_model,
+                          _abi.FLAG_OVERLAP_ENCODE if self.overlap else 0)
         # AABFT_FLAG_TOPP_IN_GEMM (include/aabft.h): run() lets the GEMM select the top-p
         # (opt-in: measured slower than selecting in the encode pass)
         self.topp_in_gemm = bool(topp_in_gemm)
@@ -149,7 +156,7 @@ class ProtectedGemm:
         if wsb == 0:
             ok(1, "aabft_workspace_bytes")
         self.ws_bytes = int(wsb)
-        self.ws = torch.empty(self.ws_bytes, dtype=torch.uint8, device=dev)
+        self.ws = torch.zeros(self.ws_bytes, dtype=torch.uint8, device=dev)
         self.enc = Encoded(self._Acs.data_ptr(), self.ld_acs, self._Bcs.data_ptr(), self.ld_bcs,
                            self.topA_val.data_ptr(), self.topA_idx.data_ptr(),
                            self.topB_val.data_ptr(), self.topB_idx.data_ptr())

@@ -57,6 +57,12 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
                              const aabft_product *out, const aabft_fault *faults,
                              int32_t nfaults, bool plain, void *ws, cudaStream_t st);
 size_t encode_ws_bytes(const aabft_config *cfg);
+// AABFT_FLAG_OVERLAP_ENCODE honoured by aabft_encode (FP64, 16 <= bs <= 64, p <= 4)
+bool encode_overlap_ok(const aabft_config *cfg);
+// 2-D FP64 TMA descriptor {inner, outer} with row pitch ld_elems (gemm_f64.cu)
+bool make_tma_2d_f64(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer,
+                     uint64_t ld_elems, uint32_t box_inner, uint32_t box_outer,
+                     CUtensorMapSwizzle sw);
 aabft_status launch_counts_sum(const aabft_counts *parts, int n, aabft_counts *out, cudaStream_t st);
 size_t gemm_f64_ws_bytes(const aabft_config *cfg);
 size_t gemm_f64_plain_ws_bytes();
@@ -230,6 +236,12 @@ __device__ __forceinline__ void tma_load_2d(void *smem_dst, const CUtensorMap *t
       " [%0], [%1, {%3, %4}], [%2];" ::"r"(smem_u32(smem_dst)),
       "l"(reinterpret_cast<uint64_t>(tm)), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
       : "memory");
+}
+
+// programmatic dependent launch: wait for the preceding grid's completion (and its memory)
+__device__ __forceinline__ void griddep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void griddep_launch_dependents() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
 }
 
 // 3D tiled TMA load global -> shared (complete_tx on an mbarrier)

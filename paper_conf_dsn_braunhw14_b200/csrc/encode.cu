@@ -21,6 +21,7 @@
 //  * Strips are double-buffered in registers (the next strip's loads are in flight during the
 //    top-p / row-sum phase).
 #include <algorithm>
+#include <atomic>
 
 #include "common.cuh"
 
@@ -429,6 +430,320 @@ __global__ void __launch_bounds__(256) topp_reduce_kernel(
   }
 }
 
+// ------------------------------------------------------------ encode overlapped with the GEMM
+// AABFT_FLAG_OVERLAP_ENCODE (FP64, bs in {16, 32, 64}, p <= 4).  The encode is HBM-bound and
+// the FP64 GEMM is DMMA-bound, and only the GEMM's checksum tiles (Ccol = Acs.B,
+// Crow = A.Bcs; the last tiles of its schedule) read the encoding, so the two run AT THE SAME
+// TIME: this kernel is a small persistent grid (one 64-thread CTA per SM, <= 64 registers,
+// ~20 KB of shared memory: it fits next to the GEMM's three CTAs per SM) that triggers its
+// dependents as soon as it starts (programmatic dependent launch); the GEMM launched after it
+// streams its data tiles at once and waits for this grid (griddepcontrol.wait) only before
+// its first checksum tile.  The paper runs its global top-p reduction "in parallel to the
+// matrix multiplication kernel"; here the whole of step 1 does.
+//
+// A unit = one block-row I of A over all K, a B unit = 64 columns of B over all K, so every
+// vector's top-p list is complete inside one CTA (no partial lists, no reduction kernel).
+// Tiles of 16 rows x 64 columns arrive by cp.async (every thread copies 16-byte chunks; rows
+// padded in shared memory) through a 2-stage ring.  The arithmetic is the sequential definition, as in the kernels above:
+// Acs -- a thread per column adds the block's rows in ascending i; Bcs -- a thread per
+// (row, block) adds the block's columns in ascending j; top-p -- branch-free pushes in
+// ascending index order, merged with the full order (key desc, index asc), so the results are
+// bit-identical to encode_ab_kernel + topp_reduce_kernel.
+constexpr int kOvR = 16, kOvC = 64;             // tile: 16 rows x 64 columns of doubles
+// padded row pitches (doubles; 16-byte multiples for cp.async): A 68 -- a half-warp of the
+// 4-lanes-per-row top-p scan touches 16 distinct bank pairs; B 66 -- the 16 row-sum threads
+// read one column with a 2-way conflict at most; every column pass is conflict-free
+constexpr int kOvPitchA = 68, kOvPitchB = 66;
+constexpr int kOvTileBytes = kOvR * kOvPitchA * 8;  // 8.5 KiB per stage
+constexpr int kOvStages = 2;
+constexpr int kOvThreads = 64;
+constexpr int kOvMaxP = 4;
+constexpr int kOvSmem = kOvStages * kOvTileBytes + 64 * kOvMaxP * 12 /*row lists*/ +
+                        2 * kOvMaxP * 12 /*warp lists*/;
+
+struct OvArgs {
+  const double *A;
+  int64_t lda;
+  const double *B;
+  int64_t ldb;
+  int64_t M, N, K;
+  int bs;
+  int nA, nB;       // units: B units (64-column groups) first, then A units (block-rows)
+  int nkt;          // B unit: 16-row tiles over K
+  int nkc, nrt;     // A unit: 64-column chunks over K x 16-row tiles per block
+  double *Acs;
+  int64_t ld_acs;
+  double *Bcs;
+  int64_t ld_bcs;
+  double *topA_v;
+  int *topA_i;
+  double *topB_v;
+  int *topB_i;
+};
+
+template <int PITCH>
+__device__ __forceinline__ double ov_at(const uint8_t *t, int r, int c) {
+  return *reinterpret_cast<const double *>(t + (r * PITCH + c) * 8);
+}
+
+__device__ __forceinline__ int ov_unit_tiles(const OvArgs &a, int u) {
+  return u < a.nB ? a.nkt : a.nkc * a.nrt;
+}
+
+// 16-byte cp.async global -> shared with zero fill beyond `bytes` (L2 only: .cg).  The loads
+// go through the SM's load/store path, not its TMA unit, which the concurrently running GEMM
+// keeps busy with its operand tiles (measured: sharing the TMA unit slowed both kernels)
+__device__ __forceinline__ void ov_cp16(void *dst, const void *src, int bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(dst)), "l"(src),
+               "r"(bytes)
+               : "memory");
+}
+
+// all 64 threads: tile `t` of unit `u` into `dst` (one 16-byte chunk per thread and row pair:
+// each warp instruction copies one contiguous 512-byte row segment)
+__device__ __forceinline__ void ov_issue(const OvArgs &a, uint8_t *dst, int u, int t) {
+  const int tid = threadIdx.x, c2 = tid & 31;
+  if (u < a.nB) {
+    const int64_t j = (int64_t)u * kOvC + 2 * c2;
+    const int cb = (int)(a.N - j < 2 ? (a.N - j > 0 ? a.N - j : 0) : 2) * 8;
+#pragma unroll
+    for (int i = 0; i < kOvR / 2; ++i) {
+      const int r = (tid >> 5) + 2 * i;
+      const int64_t k = (int64_t)t * kOvR + r;
+      const int bytes = k < a.K ? cb : 0;
+      ov_cp16(dst + (r * kOvPitchB + 2 * c2) * 8, bytes ? a.B + k * a.ldb + j : a.B, bytes);
+    }
+  } else {
+    const int I = u - a.nB, kc = t / a.nrt, rt = t % a.nrt;
+    const int64_t k = (int64_t)kc * kOvC + 2 * c2;
+    const int bytes = (int)(a.K - k < 2 ? (a.K - k > 0 ? a.K - k : 0) : 2) * 8;
+#pragma unroll
+    for (int i = 0; i < kOvR / 2; ++i) {
+      const int r = (tid >> 5) + 2 * i;
+      const int64_t row = (int64_t)I * a.bs + rt * kOvR + r;
+      ov_cp16(dst + (r * kOvPitchA + 2 * c2) * 8, bytes ? a.A + row * a.lda + k : a.A, bytes);
+    }
+  }
+  asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
+#ifdef AABFT_OV_PROBE
+// timing diagnosis: [0] first encode CTA start, [1] last encode CTA end (globaltimer, ns)
+__device__ unsigned long long g_ov_probe[2] = {~0ull, 0ull};
+__device__ __forceinline__ unsigned long long ov_gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+#endif
+
+template <int P, int BS>
+__global__ void __launch_bounds__(kOvThreads, 16) encode_overlap_kernel(const OvArgs a) {
+  // the dependent GEMM may start now: it reads the encoding only after griddepcontrol.wait
+  griddep_launch_dependents();
+#ifdef AABFT_OV_NOOP
+  return;  // timing diagnosis only (no encoding is produced)
+#endif
+#ifdef AABFT_OV_PROBE
+  if (threadIdx.x == 0) atomicMin(&g_ov_probe[0], ov_gtime());
+#endif
+  using KT = unsigned long long;
+  extern __shared__ __align__(16) uint8_t ring[];
+  KT *s_rv = reinterpret_cast<KT *>(ring + kOvStages * kOvTileBytes);  // [64 rows][P] (A)
+  int *s_ri = reinterpret_cast<int *>(s_rv + 64 * P);
+  KT *s_wv = reinterpret_cast<KT *>(s_ri + 64 * P);   // [2 warps][P] cross-warp merge
+  int *s_wi = reinterpret_cast<int *>(s_wv + 2 * P);
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int nunits = a.nA + a.nB;
+  // issue cursor (uniform over the CTA): unit iu, tile it; one commit group per stage
+  int iu = blockIdx.x, it = 0;
+  for (int s = 0; s < kOvStages; ++s) {
+    if (iu < nunits) {
+      ov_issue(a, ring + s * kOvTileBytes, iu, it);
+      if (++it == ov_unit_tiles(a, iu)) { it = 0; iu += gridDim.x; }
+    } else {
+      asm volatile("cp.async.commit_group;" ::: "memory");
+    }
+  }
+  int job = 0;
+  for (int u = blockIdx.x; u < nunits; u += gridDim.x) {
+    const int ntile = ov_unit_tiles(a, u);
+    KT cv[P];  // B: column list of column j0 + tid; A: checksum-row list over columns k0 + tid
+    int ci[P];
+    KT sv[P];  // B: list of checksum column J over this thread's rows
+    int si[P];
+    kp_init<P, KT>(cv, ci);
+    kp_init<P, KT>(sv, si);
+    double colsum = 0.0;
+    const bool isB = u < a.nB;
+    if (!isB) {
+      for (int e = tid; e < a.bs * P; e += kOvThreads) { s_rv[e] = 0; s_ri[e] = -1; }
+    }
+    for (int t = 0; t < ntile; ++t, ++job) {
+      const int s = job % kOvStages;
+      asm volatile("cp.async.wait_group %0;" ::"n"(kOvStages - 1) : "memory");
+      __syncthreads();  // every thread's chunks of stage s have landed
+      const uint8_t *tile = ring + s * kOvTileBytes;
+      if (isB) {
+        const int64_t j0 = (int64_t)u * kOvC;
+        const int k0 = t * kOvR;
+        // column top-p: thread tid owns column j0 + tid, rows in ascending k
+#pragma unroll
+        for (int r = 0; r < kOvR; ++r)
+          if (k0 + r < a.K) kp_push<P, KT>(cv, ci, Key<double>::of(ov_at<kOvPitchB>(tile, r, tid)), k0 + r);
+        // Eq 2 row checksums: thread (r, b) adds block b's bs columns of row r, ascending j
+        const int r = tid & 15, b = tid >> 4;
+        const int64_t J = j0 / BS + b;
+        if (b < kOvC / BS && k0 + r < a.K && J * BS < a.N) {
+          double sm = 0.0;
+#pragma unroll
+          for (int j8 = 0; j8 < BS; j8 += 8) {  // loads of a batch issued together
+            double x[8];
+#pragma unroll
+            for (int e = 0; e < 8; ++e) x[e] = ov_at<kOvPitchB>(tile, r, b * BS + j8 + e);
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+#ifdef AABFT_OV_NODADD  // timing diagnosis only: integer adds instead of FP64 adds
+              sm = __longlong_as_double(__double_as_longlong(sm) + __double_as_longlong(x[e]));
+#else
+              sm = sm + x[e];
+#endif
+            }
+          }
+          a.Bcs[(int64_t)(k0 + r) * a.ld_bcs + J] = sm;
+          kp_push<P, KT>(sv, si, Key<double>::of(sm), k0 + r);
+        }
+      } else {
+        const int I = u - a.nB, kc = t / a.nrt, rt = t % a.nrt;
+        const int k0 = kc * kOvC;
+        // Eq 1 column checksums: ascending i across the block's row tiles
+        if (rt == 0) colsum = 0.0;
+#pragma unroll
+        for (int r = 0; r < kOvR; ++r) {
+#ifdef AABFT_OV_NODADD
+          colsum = __longlong_as_double(__double_as_longlong(colsum) +
+                                        __double_as_longlong(ov_at<kOvPitchA>(tile, r, tid)));
+#else
+          colsum = colsum + ov_at<kOvPitchA>(tile, r, tid);
+#endif
+        }
+        // row top-p: 4 lanes per row, lane q scans columns q, q + 4, ... (ascending)
+        {
+          const int r = tid >> 2, q = tid & 3;
+          KT lv[P];
+          int li[P];
+          kp_init<P, KT>(lv, li);
+#pragma unroll
+          for (int m = 0; m < kOvC / 4; ++m) {
+            const int c = q + 4 * m;
+            const KT key = k0 + c < a.K ? Key<double>::of(ov_at<kOvPitchA>(tile, r, c)) : KT(0);
+            kp_push<P, KT>(lv, li, key, k0 + c);
+          }
+          kp_shfl_merge<P, KT>(lv, li, 1);
+          kp_shfl_merge<P, KT>(lv, li, 2);
+          if (q == 0) {  // fold into the row's running list (earlier chunks: smaller indices)
+            const int row = rt * kOvR + r;
+#pragma unroll
+            for (int e = 0; e < P; ++e) kp_insert<P, KT>(lv, li, s_rv[row * P + e], s_ri[row * P + e]);
+#pragma unroll
+            for (int e = 0; e < P; ++e) { s_rv[row * P + e] = lv[e]; s_ri[row * P + e] = li[e]; }
+          }
+        }
+        if (rt == a.nrt - 1 && k0 + tid < a.K) {
+          a.Acs[(int64_t)I * a.ld_acs + k0 + tid] = colsum;
+          kp_push<P, KT>(cv, ci, Key<double>::of(colsum), k0 + tid);
+        }
+      }
+      __syncthreads();  // stage s fully read
+      if (iu < nunits) {
+        ov_issue(a, ring + s * kOvTileBytes, iu, it);
+        if (++it == ov_unit_tiles(a, iu)) { it = 0; iu += gridDim.x; }
+      } else {
+        asm volatile("cp.async.commit_group;" ::: "memory");
+      }
+    }
+    // ---- unit epilogue: complete lists
+    if (isB) {
+      const int64_t j = (int64_t)u * kOvC + tid;
+      if (j < a.N) kp_store<double, P>(a.topB_v + j * P, a.topB_i + j * P, cv, ci);
+      // checksum column J: merge the 16 lanes (r = 0..15) of block b
+#pragma unroll
+      for (int m = 1; m < 16; m <<= 1) kp_shfl_merge<P, KT>(sv, si, m);
+      const int r = tid & 15, b = tid >> 4;
+      const int64_t J = (int64_t)u * kOvC / BS + b;
+      if (r == 0 && b < kOvC / BS && J * BS < a.N)
+        kp_store<double, P>(a.topB_v + (a.N + J) * P, a.topB_i + (a.N + J) * P, sv, si);
+    } else {
+      const int64_t I = u - a.nB;
+      for (int row = tid; row < a.bs; row += kOvThreads) {
+        KT v[P];
+        int ix[P];
+#pragma unroll
+        for (int e = 0; e < P; ++e) { v[e] = s_rv[row * P + e]; ix[e] = s_ri[row * P + e]; }
+        const int64_t gr = I * a.bs + row;
+        kp_store<double, P>(a.topA_v + gr * P, a.topA_i + gr * P, v, ix);
+      }
+      // checksum row I: merge the 64 column-owners' lists
+#pragma unroll
+      for (int m = 16; m >= 1; m >>= 1) kp_shfl_merge<P, KT>(cv, ci, m);
+      if (lane == 0) {
+#pragma unroll
+        for (int e = 0; e < P; ++e) { s_wv[(tid >> 5) * P + e] = cv[e]; s_wi[(tid >> 5) * P + e] = ci[e]; }
+      }
+      __syncthreads();
+      if (tid == 0) {
+#pragma unroll
+        for (int e = 0; e < P; ++e) kp_insert<P, KT>(cv, ci, s_wv[P + e], s_wi[P + e]);
+        kp_store<double, P>(a.topA_v + (a.M + I) * P, a.topA_i + (a.M + I) * P, cv, ci);
+      }
+      __syncthreads();  // s_rv / s_wv free for the next unit
+    }
+  }
+  asm volatile("cp.async.wait_all;" ::: "memory");
+#ifdef AABFT_OV_PROBE
+  if (threadIdx.x == 0) atomicMax(&g_ov_probe[1], ov_gtime());
+#endif
+}
+
+template <int P, int BS>
+aabft_status run_encode_overlap(const aabft_config *cfg, const double *A, int64_t lda,
+                                const double *B, int64_t ldb, const aabft_encoded *out,
+                                cudaStream_t st) {
+  const int64_t M = cfg->M, N = cfg->N, K = cfg->K;
+  OvArgs a{};
+  a.A = A; a.lda = lda; a.B = B; a.ldb = ldb;
+  a.M = M; a.N = N; a.K = K; a.bs = cfg->bs;
+  a.nB = (int)((N + kOvC - 1) / kOvC);
+  a.nA = (int)(M / cfg->bs);
+  a.nkt = (int)((K + kOvR - 1) / kOvR);
+  a.nkc = (int)((K + kOvC - 1) / kOvC);
+  a.nrt = cfg->bs / kOvR;
+  a.Acs = static_cast<double *>(out->Acs); a.ld_acs = out->ld_acs;
+  a.Bcs = static_cast<double *>(out->Bcs); a.ld_bcs = out->ld_bcs;
+  a.topA_v = out->topA_val; a.topA_i = out->topA_idx;
+  a.topB_v = out->topB_val; a.topB_i = out->topB_idx;
+  static std::atomic<int> sms_dev[64];  // per instantiation and device
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int sms = sms_dev[dev & 63].load(std::memory_order_relaxed);
+  if (!sms) {
+    if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
+      return check_launch("encode_overlap SM count");
+    for (const void *fn : {(const void *)encode_overlap_kernel<P, BS>}) {
+      if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kOvSmem) != cudaSuccess ||
+          cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout,
+                               cudaSharedmemCarveoutMaxShared) != cudaSuccess)
+        return check_launch("encode_overlap attributes");
+    }
+    sms_dev[dev & 63].store(sms, std::memory_order_relaxed);
+  }
+  const int units = a.nA + a.nB;
+  const int grid = std::min(units, sms);  // one CTA per SM, next to the GEMM's CTAs
+  encode_overlap_kernel<P, BS><<<grid, kOvThreads, kOvSmem, st>>>(a);
+  next_launch();
+  return check_launch("aabft_encode (overlapped)");
+}
+
 // workspace: [A partial values][A partial indices][B values][B indices]
 struct EncWs {
   double *pva, *pvb;
@@ -524,6 +839,15 @@ aabft_status dispatch_p(const aabft_config *cfg, const void *A, int64_t lda, con
 
 }  // namespace
 
+#ifdef AABFT_OV_PROBE
+extern "C" int aabft_debug_ov_probe(unsigned long long *out2) {
+  cudaMemcpyFromSymbol(out2, g_ov_probe, 16);
+  const unsigned long long init[2] = {~0ull, 0ull};
+  cudaMemcpyToSymbol(g_ov_probe, init, 16);
+  return 0;
+}
+#endif
+
 size_t encode_ws_bytes(const aabft_config *cfg) {
   const size_t p = (size_t)cfg->p;
   const size_t ncha = (size_t)enc_a_chunks(cfg->K), nchb = (size_t)enc_b_chunks(cfg->K);
@@ -532,8 +856,23 @@ size_t encode_ws_bytes(const aabft_config *cfg) {
          r256e(rb * nchb * p * 4);
 }
 
+bool encode_overlap_ok(const aabft_config *cfg) {
+  return (cfg->flags & AABFT_FLAG_OVERLAP_ENCODE) && cfg->dtype == AABFT_F64 &&
+         cfg->bs >= 16 && cfg->bs <= 64 && cfg->p <= kOvMaxP &&
+         !((cfg->flags & AABFT_FLAG_TOPP_IN_GEMM) && gemm_f64_topp_ok(cfg));
+}
+
 aabft_status launch_encode(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
                            int64_t ldb, const aabft_encoded *out, void *ws, cudaStream_t st) {
+  if (encode_overlap_ok(cfg) && A && B && out->topA_val && out->topB_val) {
+    const double *a = static_cast<const double *>(A), *b = static_cast<const double *>(B);
+#define AABFT_OV_CASE(PP, BB) \
+  if (cfg->p == PP && cfg->bs == BB) return run_encode_overlap<PP, BB>(cfg, a, lda, b, ldb, out, st);
+#define AABFT_OV_BS(PP) AABFT_OV_CASE(PP, 16) AABFT_OV_CASE(PP, 32) AABFT_OV_CASE(PP, 64)
+    AABFT_OV_BS(1) AABFT_OV_BS(2) AABFT_OV_BS(3) AABFT_OV_BS(4)
+#undef AABFT_OV_BS
+#undef AABFT_OV_CASE
+  }
   if (cfg->dtype == AABFT_F64) return dispatch_p<double>(cfg, A, lda, B, ldb, out, ws, st);
   return dispatch_p<float>(cfg, A, lda, B, ldb, out, ws, st);
 }

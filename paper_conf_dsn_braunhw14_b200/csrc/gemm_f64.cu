@@ -87,8 +87,11 @@ constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 constexpr int MAXF = 64;                    // faults per 64x64 tile kept in smem (one per 8x8 block)
 constexpr int BOOK = 128;                   // barriers, counters, cursor
 constexpr int SUMBUF = 4 * 64 * 8;           // BS = 64 epilogue exchange (kCtaSums)
-constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 1024 /*align*/ + BOOK +
-                           MAXF * (int)sizeof(aabft_fault) + SUMBUF;
+// [ring][bookkeeping][BS = 64 sum exchange][fault list: FAULTS instantiation only -- the
+// production kernel leaves ~23 KB per SM free for the overlapped encode's CTA]
+constexpr int SMEM_PROD = STAGES * STAGE_BYTES + 1024 /*align*/ + BOOK + SUMBUF;
+constexpr int SMEM_FAULTS = SMEM_PROD + MAXF * (int)sizeof(aabft_fault);
+constexpr int smem_bytes(bool faults) { return faults ? SMEM_FAULTS : SMEM_PROD; }
 constexpr int GROUP_M = AABFT_F64_GROUP_M;
 constexpr int kMaxCtas = 1024;              // >= resident CTAs; sizes the split-K partial slots
 constexpr int ACC = MT * NT * 4;            // accumulators per thread
@@ -387,6 +390,16 @@ __device__ __forceinline__ void issue_stage(const GemmArgs &a, const CUtensorMap
   tma_load_2d(sa, tl.type == 1 ? tmAcs : tmA, bar, k, tl.m0);
 }
 
+#ifdef AABFT_OV_PROBE
+// timing diagnosis: [0] first CTA start, [1] last producer end, [2] latest encode-wait return
+__device__ unsigned long long g_gemm_probe[3] = {~0ull, 0ull, 0ull};
+__device__ __forceinline__ unsigned long long gemm_gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+#endif
+
 template <bool FAULTS, int TP>
 __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
     gemm_f64_kernel(const __grid_constant__ CUtensorMap tmA,
@@ -402,9 +415,9 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
   uint64_t *empty = full + STAGES;
   int *s_nf = reinterpret_cast<int *>(empty + STAGES);
   static_assert(16 * STAGES + 8 <= BOOK, "bookkeeping fits");
-  aabft_fault *s_f = reinterpret_cast<aabft_fault *>(smem + STAGES * STAGE_BYTES + BOOK);
-  double *s_csum = reinterpret_cast<double *>(s_f + MAXF);  // [2][64] column parts (row halves)
-  double *s_rsum = s_csum + 128;                              // [2][64] row parts (column halves)
+  double *s_csum = reinterpret_cast<double *>(smem + STAGES * STAGE_BYTES + BOOK);  // [2][64] column parts
+  double *s_rsum = s_csum + 128;                                                   // [2][64] row parts
+  aabft_fault *s_f = reinterpret_cast<aabft_fault *>(s_csum + 256);  // FAULTS only
 
   // warp roles: the producer is the CTA's last warp (AABFT_F64_PROD_FIRST: its first);
   // mtid / mwarp index the 4 MMA warps
@@ -422,6 +435,9 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
   const int my_dp = min(args.waves, ((int)args.ntiles - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x);
   const int njobs = my_dp * args.nk + (int)(sk1 - sk0);
 
+#ifdef AABFT_OV_PROBE
+  if (threadIdx.x == 0) atomicMin(&g_gemm_probe[0], gemm_gtime());
+#endif
   if (threadIdx.x == 0) {
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&full[s], 1);
@@ -443,6 +459,10 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
     }
     int tile = -1, kt = 0;
     Tile tl{0, 0, 0};
+    bool enc_ready = false;  // griddepcontrol.wait done (AABFT_FLAG_OVERLAP_ENCODE)
+#ifdef AABFT_OV_PROBE
+    unsigned long long first_cs_wait_end = 0;
+#endif
     constexpr int SP = TP > 0 ? TP : 1;
     TopScan<SP> sc;
     sc.tile = -1;
@@ -457,13 +477,34 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
       if (jn >= STAGES) mbar_wait(&empty[s], (uint32_t)(((jn / STAGES) & 1) ^ 1));
       uint8_t *sa = smem + s * STAGE_BYTES;
       const int k = kt * BK;
-      if (lane == 0) issue_stage(args, &tmA, &tmAcs, &tmB, &tmBcs, sa, &full[s], tl, k);
+      if (lane == 0) {
+        // checksum tiles read Acs / Bcs, which a programmatically-dependent launch may still
+        // be producing: wait for the preceding grid (no-op without PDL).  Data tiles read only
+        // A and B and never wait.
+        if (tl.type != 0 && !enc_ready) {
+          griddep_wait();
+          enc_ready = true;
+#ifdef AABFT_OV_PROBE
+          first_cs_wait_end = gemm_gtime();
+#endif
+        }
+        issue_stage(args, &tmA, &tmAcs, &tmB, &tmBcs, sa, &full[s], tl, k);
+      }
       __syncwarp();
       if (TP > 0 && jn >= kScanLag) scan_job<SP>(args, smem, full, jn - kScanLag, njobs, sk0, sc, lane);
     }
     if (TP > 0)
       for (int js = max(0, njobs - kScanLag); js < njobs; ++js)
         scan_job<SP>(args, smem, full, js, njobs, sk0, sc, lane);
+    // the grid never completes before the grid it depends on (stream order is kept for the
+    // kernels after it, e.g. aabft_check reading the top-p tables)
+    if (lane == 0 && !enc_ready) griddep_wait();
+#ifdef AABFT_OV_PROBE
+    if (lane == 0) {
+      atomicMax(&g_gemm_probe[1], gemm_gtime());           // last producer done
+      atomicMax(&g_gemm_probe[2], first_cs_wait_end);      // latest return from the encode wait
+    }
+#endif
     return;
   }
 
@@ -864,6 +905,21 @@ bool make_map(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer, 
 
 }  // namespace
 
+#ifdef AABFT_OV_PROBE
+extern "C" int aabft_debug_gemm_probe(unsigned long long *out3) {
+  cudaMemcpyFromSymbol(out3, g_gemm_probe, 24);
+  const unsigned long long init[3] = {~0ull, 0ull, 0ull};
+  cudaMemcpyToSymbol(g_gemm_probe, init, 24);
+  return 0;
+}
+#endif
+
+bool make_tma_2d_f64(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer,
+                     uint64_t ld_elems, uint32_t box_inner, uint32_t box_outer,
+                     CUtensorMapSwizzle sw) {
+  return make_map(m, base, inner, outer, ld_elems, box_inner, box_outer, sw);
+}
+
 static size_t r256z(size_t b) { return (b + 255) / 256 * 256; }
 // [split-K accumulator partials][flags][top-p flags][top-p partial values][indices][R planes]
 static size_t flags_off() { return r256z((size_t)kMaxCtas * ACC * THREADS * sizeof(double)); }
@@ -914,10 +970,12 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
       for (int tp = 0; tp <= kTpMaxP; ++tp) {
         const void *fn = kernel_for(f != 0, tp);
         int n = 0;
-        if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES) !=
-            cudaSuccess)
+        if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes(f != 0)) !=
+                cudaSuccess ||
+            cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                 cudaSharedmemCarveoutMaxShared) != cudaSuccess)
           return check_launch("gemm_f64 smem attribute");
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, CTA_THREADS, SMEM_BYTES) !=
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, CTA_THREADS, smem_bytes(f != 0)) !=
                 cudaSuccess || n < 1)
           return check_launch("gemm_f64 occupancy");
         per_sm = std::min(per_sm, n);
@@ -1003,19 +1061,31 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
     }
   }
   if (total > 0) {
-    if (a.sk_iters > 0 && cudaMemsetAsync(a.flags, 0, 2 * kMaxCtas * sizeof(int), st) != cudaSuccess)
+    // AABFT_FLAG_OVERLAP_ENCODE (protected product): a programmatic dependent launch of the
+    // preceding aabft_encode; the flag words are zero on entry by contract (workspace zeroed
+    // once, every launch re-arms the words it used), so no reset sits between the two grids
+    const bool overlap = !plain && (cfg->flags & AABFT_FLAG_OVERLAP_ENCODE);
+    if (!overlap && a.sk_iters > 0 &&
+        cudaMemsetAsync(a.flags, 0, 2 * kMaxCtas * sizeof(int), st) != cudaSuccess)
       return check_launch("gemm_f64 flag reset");
     // split-tile owners spin on flags set by later CTAs: with a stream-K tail the launch is
     // COOPERATIVE, so a grid that cannot be co-resident (other kernels, MPS, green contexts)
-    // waits for room or fails instead of hanging
+    // waits for room or fails instead of hanging.  Overlapped with the encode it
+    // is a plain launch: the encode grid it may share the GPU with never waits on the GEMM,
+    // so every GEMM CTA becomes resident at the latest when the encode's CTAs exit.
     cudaLaunchConfig_t lc = {};
     lc.gridDim = dim3((unsigned)grid);
     lc.blockDim = dim3(CTA_THREADS);
-    lc.dynamicSmemBytes = SMEM_BYTES;
+    lc.dynamicSmemBytes = smem_bytes(a.nfaults > 0);
     lc.stream = st;
     cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeCooperative;
-    attr[0].val.cooperative = a.sk_iters > 0 ? 1 : 0;
+    if (overlap) {
+      attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+      attr[0].val.programmaticStreamSerializationAllowed = 1;
+    } else {
+      attr[0].id = cudaLaunchAttributeCooperative;
+      attr[0].val.cooperative = a.sk_iters > 0 ? 1 : 0;
+    }
     lc.attrs = attr;
     lc.numAttrs = 1;
     void *params[] = {&tA, &tAcs, &tB, &tBcs, &a};
