@@ -104,6 +104,13 @@ typedef struct {
  * DMMA instructions, which stretches the co-resident encode 7x and costs the GEMM more than
  * the serial encode takes. */
 #define AABFT_FLAG_OVERLAP_ENCODE 4
+/* AABFT_FLAG_CHECK_CORRECTS: aabft_check also corrects every block it locates as SINGLE, in the
+ * same kernel (Alg 2 classifies and corrects per block): the block's report leaves
+ * the check as AABFT_BLK_CORRECTED or AABFT_BLK_UNCORRECTABLE (the correction is re-verified
+ * exactly as aabft_correct does), the counters include the corrections, and a following
+ * aabft_correct finds nothing left to do.  Without the flag aabft_check only classifies and
+ * locates (AABFT_BLK_SINGLE) and aabft_correct corrects. */
+#define AABFT_FLAG_CHECK_CORRECTS 8
 
 /* Output of aabft_encode.  Acs: (M/bs) x K, ld_acs >= K.  Bcs: K x (N/bs), ld_bcs >= N/bs.
  * topA_val/topA_idx: (M + M/bs) x p -- data rows 0..M-1, then checksum rows; |value|
@@ -196,7 +203,11 @@ typedef struct {
 
 /* Bytes of device workspace needed by aabft_encode / aabft_gemm / aabft_gemm_plain /
  * aabft_check (one buffer serves all of them; 256-byte aligned; contents need no
- * initialisation).  Returns 0 on an invalid config. */
+ * initialisation -- except under AABFT_FLAG_OVERLAP_ENCODE, see there).  A fused aabft_check
+ * must get the workspace of the aabft_gemm that produced its product: that GEMM zeroes the
+ * check's counter accumulator (the workspace's last 256 bytes), the check's CTAs add into it
+ * and its last CTA moves the totals to *counts and re-arms it.  Returns 0 on an invalid
+ * config. */
 size_t aabft_workspace_bytes(const aabft_config *cfg);
 
 /* Step 1 (Alg 1).  A (lda >= K) or B (ldb >= N) may be NULL to encode only the
@@ -241,8 +252,8 @@ aabft_status aabft_gemm_plain(const aabft_config *cfg, const void *A, int64_t ld
                               const void *B, int64_t ldb, void *C, int64_t ldc, void *ws,
                               size_t ws_bytes, void *stream);
 
-/* Step 3 (Alg 2; Eq 4-6).  Writes (M/bs)*(N/bs) reports and zeroes then fills
- * *counts (device).  Reference sums are in double (reading R12): unfused (prod->Rcol/Rrow
+/* Step 3 (Alg 2; Eq 4-6).  Writes (M/bs)*(N/bs) reports and overwrites *counts
+ * (device) with this check's totals (AABFT_FLAG_CHECK_CORRECTS: also corrects SINGLE blocks).  Reference sums are in double (reading R12): unfused (prod->Rcol/Rrow
  * NULL, or FP32, or bs > 64) they re-sum C from memory in sequential ascending order -- the
  * paper's check kernel; fused they are the GEMM epilogue's sums of the registers it
  * stored (fixed shuffle-tree order, parity by tolerance) -- which sees every fault inside the

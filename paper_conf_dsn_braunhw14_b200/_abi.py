@@ -20,6 +20,7 @@ STATUS_NAMES = {0: "CLEAN", 1: "CORRECTED", 2: "CHECKSUM_ONLY", 3: "UNCORRECTABL
 FLAG_TOPP_IN_GEMM = 1  # include/aabft.h AABFT_FLAG_TOPP_IN_GEMM
 FLAG_GEMM_HALF_GRID = 2  # AABFT_FLAG_GEMM_HALF_GRID
 FLAG_OVERLAP_ENCODE = 4  # AABFT_FLAG_OVERLAP_ENCODE
+FLAG_CHECK_CORRECTS = 8  # AABFT_FLAG_CHECK_CORRECTS
 COUNT_NAMES = ("blocks", "clean", "corrected", "checksum_only", "uncorrectable",
                "checks_rounding", "checks_tolerable", "checks_critical")
 EXPORTED = ("aabft_workspace_bytes", "aabft_encode", "aabft_bound", "aabft_bound_elements",

@@ -131,6 +131,9 @@ class ProtectedGemm:
         self.topp_in_gemm = bool(topp_in_gemm)
         self.cfg_defer = Config(_dtype_code(dtype), bs, M, N, K, p, t, omega, fma_model,
                                 _abi.FLAG_TOPP_IN_GEMM)
+        # AABFT_FLAG_CHECK_CORRECTS: run(correct=True) corrects inside the check kernel
+        self.cfg_cc = Config(_dtype_code(dtype), bs, M, N, K, p, t, omega, fma_model,
+                             self.cfg.flags | _abi.FLAG_CHECK_CORRECTS)
         self._topp_pending = False
         dev, dt = self.device, dtype
         nI, nJ = M // bs, N // bs
@@ -221,8 +224,11 @@ class ProtectedGemm:
                             nfaults, self.ws.data_ptr(), self.ws_bytes, _stream_ptr(stream)),
            "aabft_gemm")
 
-    def check(self, stream=None):
-        ok(lib().aabft_check(C.byref(self.cfg), C.byref(self.enc), C.byref(self.prod),
+    def check(self, stream=None, correct: bool = False):
+        """Step 3; correct=True also corrects the located single errors in the same kernel
+        (AABFT_FLAG_CHECK_CORRECTS), which makes correct() unnecessary."""
+        cfg = self.cfg_cc if correct else self.cfg
+        ok(lib().aabft_check(C.byref(cfg), C.byref(self.enc), C.byref(self.prod),
                              self.reports.data_ptr(), self.counts.data_ptr(), self.ws.data_ptr(),
                              self.ws_bytes, _stream_ptr(stream)), "aabft_check")
 
@@ -320,16 +326,15 @@ class ProtectedGemm:
         return self.result()
 
     def run(self, A, B, *, faults=None, correct: bool = True, stream=None) -> Result:
-        """encode -> gemm -> check -> correct, all enqueued on one stream."""
+        """encode -> gemm -> check + correct, all enqueued on one stream; the
+        correction of located single errors runs inside the check kernel."""
         self._check_operand(A, self.M, self.K, "A")
         self._check_operand(B, self.K, self.N, "B")
         fbuf = faults if isinstance(faults, torch.Tensor) else make_faults(faults, self.device)
         nf = 0 if fbuf is None else fbuf.numel() // 48
         self.encode(A, B, stream, defer=self.topp_in_gemm)
         self.gemm(A, B, fbuf, nf, stream)
-        self.check(stream)
-        if correct:
-            self.correct(stream)
+        self.check(stream, correct=correct)  # correction fused into the check kernel
         return self.result()
 
     def capture(self, A, B, *, correct: bool = True):

@@ -117,6 +117,13 @@ static void *gemm_ws(const aabft_config *c, void *ws) {
   return static_cast<char *>(ws) + front_ws_bytes(c);
 }
 
+// the check's counter accumulator: the workspace's trailing 256 bytes (10 words used),
+// zeroed by aabft_gemm of the protected product and re-armed by the check's last CTA
+static unsigned long long *check_acc(const aabft_config *c, void *ws) {
+  return reinterpret_cast<unsigned long long *>(static_cast<char *>(ws) + front_ws_bytes(c) +
+                                                r256(gemm_ws_bytes(c)));
+}
+
 static bool pitch_ok(const aabft_config *c, const void *p, int64_t ld) {
   return aligned16(p) && ((size_t)ld * elem_size(c)) % 16 == 0;
 }
@@ -257,8 +264,10 @@ static aabft_status gemm_common(const aabft_config *cfg, const void *A, int64_t 
   if ((s = device_ok()) != AABFT_OK) return s;
   if (cfg->dtype == AABFT_F64)
     return launch_gemm_f64(cfg, A, lda, B, ldb, enc, out, plain ? nullptr : faults, plain ? 0 : nfaults, plain,
-                           plain ? ws : gemm_ws(cfg, ws), (cudaStream_t)stream);
-  return launch_gemm_f32(cfg, A, lda, B, ldb, enc, out, plain ? nullptr : faults, plain ? 0 : nfaults, plain, (cudaStream_t)stream);
+                           plain ? ws : gemm_ws(cfg, ws), plain ? nullptr : check_acc(cfg, ws),
+                           (cudaStream_t)stream);
+  return launch_gemm_f32(cfg, A, lda, B, ldb, enc, out, plain ? nullptr : faults, plain ? 0 : nfaults, plain,
+                         plain ? nullptr : check_acc(cfg, ws), (cudaStream_t)stream);
 }
 
 aabft_status aabft_gemm(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
@@ -303,8 +312,9 @@ aabft_status aabft_check(const aabft_config *cfg, const aabft_encoded *enc,
     set_error("check (fused): the aabft_gemm workspace is required");
     return AABFT_EWORKSPACE;
   }
+  // fused: the GEMM's workspace, whose check accumulator that GEMM zeroed (no memset here)
   return launch_check(cfg, enc, prod, reports, counts, fused ? gemm_ws(cfg, ws) : nullptr,
-                      (cudaStream_t)stream);
+                      fused ? check_acc(cfg, ws) : nullptr, (cudaStream_t)stream);
   AABFT_GUARD_END
 }
 
@@ -369,7 +379,8 @@ aabft_status aabft_check_ext(const aabft_config *cfg, const aabft_product *prod,
     return AABFT_EWORKSPACE;
   }
   return launch_check_ext(cfg, prod, eps_col, eps_row, eps_fixed, reports, counts,
-                          fused ? gemm_ws(cfg, ws) : nullptr, (cudaStream_t)stream);
+                          fused ? gemm_ws(cfg, ws) : nullptr, fused ? check_acc(cfg, ws) : nullptr,
+                          (cudaStream_t)stream);
   AABFT_GUARD_END
 }
 
@@ -586,6 +597,7 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
       cb.M = mi;
       cb.N = nj;
       if (two) cb.flags |= AABFT_FLAG_GEMM_HALF_GRID;
+      cb.flags |= AABFT_FLAG_CHECK_CORRECTS;  // correction inside the check kernel
       const bool second = two && (nblk & 1);
       cudaStream_t cs = second ? hp.c2 : st;
       void *ws = base + (second ? a.oWs2 : a.oWs);
@@ -624,7 +636,6 @@ aabft_status aabft_protected_gemm_host(const aabft_config *cfg, const void *A_ho
       aabft_counts *cnt = cnt_blocks + nblk;
       if ((s = aabft_gemm(&cb, Ai, a.lda, Bj, a.ldb, &enc, &prod, nullptr, 0, ws, wsb, cs)) != AABFT_OK) return s;
       if ((s = aabft_check(&cb, &enc, &prod, rep, cnt, ws, wsb, cs)) != AABFT_OK) return s;
-      if ((s = aabft_correct(&cb, &enc, &prod, rep, cnt, cs)) != AABFT_OK) return s;
       // device -> host of the finished (corrected) C block on the copy-out stream
       cudaEventRecord(evC[nblk], cs);
       mark(cs, "block done", i, j);

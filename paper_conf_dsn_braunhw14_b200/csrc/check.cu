@@ -156,6 +156,11 @@ struct CheckArgs {
   const double *eps_col;  // (M/bs) x N dense, or NULL
   const double *eps_row;  // M x (N/bs) dense, or NULL
   double eps_fixed;
+  // counters: CTAs add into the workspace accumulator `acc` (zeroed by aabft_gemm, re-armed by
+  // the last CTA, which writes the totals to `cnt`), so no memset sits between the GEMM and
+  // the check; NULL = add straight into `cnt` after a memset (no workspace given)
+  unsigned long long *acc;  // [9]: n[8], max_ratio bits; [9]: CTA ticket
+  int correct;              // AABFT_FLAG_CHECK_CORRECTS: correct SINGLE blocks in place
 };
 
 // Bound of column check (I, j) / row check (i, J): the A-ABFT bound from the top-p tables, or
@@ -216,6 +221,70 @@ __device__ __forceinline__ void finish_block(const CheckArgs &a, int64_t blk, in
                           (unsigned long long)__double_as_longlong(br));
 }
 
+// Alg 2's correction of one SINGLE block (row i, column j located by the check): returns
+// AABFT_BLK_CORRECTED, or AABFT_BLK_UNCORRECTABLE when the re-verified row still fails
+template <typename T, int P, bool EXT>
+__device__ __forceinline__ uint8_t correct_block(const CheckArgs &a, const BoundParams &bp, T *C, int64_t blk,
+                                 int64_t i, int64_t j) {
+  const int bs = a.bs;
+  const int64_t nJ = a.N / bs;
+  const int64_t I = blk / nJ, J = blk % nJ;
+  // c_ij <- Ccol[I][j] - sum_{i' != i} c_i'j  (reading R15; double, ascending i')
+  double v = (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
+  for (int64_t ii = I * bs; ii < I * bs + bs; ++ii)
+    if (ii != i) v = v - (double)C[ii * a.ldc + j];
+  C[i * a.ldc + j] = (T)v;
+  // re-verify row i
+  double ref = 0.0;
+  for (int64_t jj = J * bs; jj < J * bs + bs; ++jj) ref = ref + (double)C[i * a.ldc + jj];
+  const double d = ref - (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
+  const Bound b = row_bound<EXT, P>(a, bp, i, J);
+  if (a.Rcol) {
+    // fused check: the epilogue reference sums still describe the faulty element; refresh
+    // the two that pass through (i, j) from the corrected C so a later aabft_check of the
+    // same product sees the corrected state (ascending order, double)
+    double rc = 0.0;
+    for (int64_t ii = I * bs; ii < I * bs + bs; ++ii) rc = rc + (double)C[ii * a.ldc + j];
+    const_cast<double *>(a.Rcol)[I * a.N + j] = rc;
+    const_cast<double *>(a.Rrow)[i * nJ + J] = ref;
+  }
+  return fabs(d) <= b.eps ? (uint8_t)AABFT_BLK_CORRECTED : (uint8_t)AABFT_BLK_UNCORRECTABLE;
+}
+
+// Block-verdict epilogue of both check kernels: AABFT_FLAG_CHECK_CORRECTS corrects a SINGLE
+// block right here (the CTA owns the whole block; Alg 2 classifies and corrects in one kernel,
+// P:L380-393), so the step needs no separate correction launch.
+template <typename T, int P, bool EXT>
+__device__ __forceinline__ uint8_t maybe_correct(const CheckArgs &a, const BoundParams &bp,
+                                                 uint8_t status, int64_t blk, int row, int col) {
+  if (!a.correct || status != AABFT_BLK_SINGLE) return status;
+  return correct_block<T, P, EXT>(a, bp, static_cast<T *>(const_cast<void *>(a.C)), blk, row, col);
+}
+
+// CTA counters (s_n[8], s_mr: float bits) -> device totals.  With a workspace accumulator the
+// CTAs add into it and the LAST CTA (ticket) moves the totals into `cnt` and re-arms the
+// accumulator (threadfence-reduction pattern); otherwise straight atomics into the zeroed cnt.
+__device__ __forceinline__ void publish_counts(const CheckArgs &a, const unsigned long long *s_n,
+                                               unsigned s_mr, int tid) {
+  unsigned long long *dst = a.acc ? a.acc : reinterpret_cast<unsigned long long *>(a.cnt->n);
+  if (tid < 8 && s_n[tid]) atomicAdd(dst + tid, s_n[tid]);
+  if (tid == 8 && s_mr) atomicMax(dst + 8, (unsigned long long)__double_as_longlong((double)__uint_as_float(s_mr)));
+  if (!a.acc) return;
+  __shared__ bool s_last;
+  __threadfence();
+  __syncthreads();
+  if (tid == 0) {
+    const unsigned total = gridDim.x * gridDim.y;
+    s_last = atomicAdd(reinterpret_cast<unsigned *>(a.acc + 9), 1u) == total - 1;
+  }
+  __syncthreads();
+  if (s_last) {
+    __threadfence();
+    if (tid < 9) reinterpret_cast<unsigned long long *>(a.cnt)[tid] = atomicExch(a.acc + tid, 0ull);
+    if (tid == 0) atomicExch(reinterpret_cast<unsigned *>(a.acc + 9), 0u);
+  }
+}
+
 // --------------------------------------------------------------------------- fused check
 // The GEMM epilogue already produced the reference sums (Rcol, Rrow); compare them with the
 // carried checksums: 2*bs checks per block, no pass over C.  Latency-bound work, so it is laid
@@ -242,8 +311,8 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
   const int64_t nJ = a.N / bs;
   if (tid < 8) s_n[tid] = 0ull;
   if (tid == 8) s_mr = 0u;
-  unsigned long long my_n[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-  int cls_tot[3] = {0, 0, 0};
+  unsigned my_n[5] = {0, 0, 0, 0, 0};  // blocks, clean, corrected, checksum-only, uncorrectable
+  unsigned cls0 = 0, cls1 = 0, cls2 = 0;  // checks per class (registers, not an indexed array)
   float mr = 0.f;
   const int cseg = bs < 32 ? bs : 32;  // lanes sharing one block among the column checks
   for (int64_t u = blockIdx.x; u < nunits; u += gridDim.x) {
@@ -294,7 +363,7 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
       if (hc) {
         const double d = refc - carc;
         const int cl = classify(d, bc);
-        cls_tot[cl] += 1;
+        cls0 += cl == 0; cls1 += cl == 1; cls2 += cl == 2;
         if (cl) {
           atomicMax(&s_worst[Jc], cl);
           if (cl == 2) { atomicAdd(&s_nc[Jc], 1); s_col[Jc] = (int)j; }
@@ -314,7 +383,7 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
       if (hr) {
         const double d = refr - carr;
         const int cl = classify(d, brw);
-        cls_tot[cl] += 1;
+        cls0 += cl == 0; cls1 += cl == 1; cls2 += cl == 2;
         if (cl) {
           atomicMax(&s_worst[Jr], cl);
           if (cl == 2) { atomicAdd(&s_nr[Jr], 1); s_row[Jr] = (int)i; }
@@ -350,15 +419,27 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
       my_n[3] += status == AABFT_BLK_CHECKSUM_ONLY;
       my_n[4] += status == AABFT_BLK_UNCORRECTABLE;
       mr = fmaxf(mr, br);
+      s_nc[tid] = status == AABFT_BLK_SINGLE ? 1 : 0;  // (slot reused: SINGLE marker)
+    }
+    __syncthreads();
+    // AABFT_FLAG_CHECK_CORRECTS: correct this unit's SINGLE blocks (a separate phase, so the
+    // rare correction code does not add to the register pressure of the check above)
+    if (a.correct && tid < JB && J0 + tid < nJ && s_nc[tid]) {
+      const int64_t blk = I * nJ + J0 + tid;
+      const uint8_t st = correct_block<T, P, EXT>(a, bp, static_cast<T *>(const_cast<void *>(a.C)),
+                                                  blk, s_row[tid], s_col[tid]);
+      a.rep[blk].status = st;
+      my_n[2] += st == AABFT_BLK_CORRECTED;
+      my_n[4] += st == AABFT_BLK_UNCORRECTABLE;
     }
     __syncthreads();  // the per-block slots are re-initialised by the next unit
   }
   // ---- CTA aggregation: warp reductions (REDUX), then one global atomic per non-zero counter
   // (per-thread totals are far below 2^32: a CTA handles a few units of 2 x 256 checks)
-  my_n[5] = cls_tot[0]; my_n[6] = cls_tot[1]; my_n[7] = cls_tot[2];
+  const unsigned tot[8] = {my_n[0], my_n[1], my_n[2], my_n[3], my_n[4], cls0, cls1, cls2};
   unsigned wn[8];
 #pragma unroll
-  for (int c = 0; c < 8; ++c) wn[c] = __reduce_add_sync(0xffffffffu, (unsigned)my_n[c]);
+  for (int c = 0; c < 8; ++c) wn[c] = __reduce_add_sync(0xffffffffu, tot[c]);
   const unsigned wmr = __reduce_max_sync(0xffffffffu, __float_as_uint(mr));
   if (lane == 0) {
 #pragma unroll
@@ -367,10 +448,7 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
     if (wmr) atomicMax(&s_mr, wmr);
   }
   __syncthreads();
-  if (tid < 8 && s_n[tid]) atomicAdd(reinterpret_cast<unsigned long long *>(a.cnt->n) + tid, s_n[tid]);
-  if (tid == 8 && s_mr)
-    atomicMax(reinterpret_cast<unsigned long long *>(&a.cnt->max_ratio),
-              (unsigned long long)__double_as_longlong((double)__uint_as_float(s_mr)));
+  publish_counts(a, s_n, s_mr, tid);
 }
 
 // --------------------------------------------------------------------------- streaming check
@@ -483,11 +561,13 @@ __global__ void __launch_bounds__(CW) check_stream_kernel(CheckArgs a, BoundPara
     rep.col = status == AABFT_BLK_SINGLE ? s_col[c] : -1;
     mr = __uint_as_float(s_rmax[c]);
     rep.max_ratio = mr;
+    rep.status = maybe_correct<T, P, EXT>(a, bp, status, I * nJ + j0 / bs + c, rep.row, rep.col);
     a.rep[I * nJ + j0 / bs + c] = rep;
     my_n[0] = 1;
     my_n[1] = status == AABFT_BLK_CLEAN;
+    my_n[2] = rep.status == AABFT_BLK_CORRECTED;
     my_n[3] = status == AABFT_BLK_CHECKSUM_ONLY;
-    my_n[4] = status == AABFT_BLK_UNCORRECTABLE;
+    my_n[4] = rep.status == AABFT_BLK_UNCORRECTABLE;
   }
   my_n[5] = cls_tot[0]; my_n[6] = cls_tot[1]; my_n[7] = cls_tot[2];
 #pragma unroll
@@ -503,10 +583,7 @@ __global__ void __launch_bounds__(CW) check_stream_kernel(CheckArgs a, BoundPara
     if (mr > 0.f) atomicMax(&s_mr, __float_as_uint(mr));
   }
   __syncthreads();
-  if (c < 8 && s_n[c]) atomicAdd(reinterpret_cast<unsigned long long *>(a.cnt->n) + c, s_n[c]);
-  if (c == 8 && s_mr)
-    atomicMax(reinterpret_cast<unsigned long long *>(&a.cnt->max_ratio),
-              (unsigned long long)__double_as_longlong((double)__uint_as_float(s_mr)));
+  publish_counts(a, s_n, s_mr, c);
 }
 
 // --------------------------------------------------------------------------- correct
@@ -518,34 +595,10 @@ __global__ void correct_kernel(CheckArgs a, BoundParams bp, T *C) {
        blk += (int64_t)gridDim.x * blockDim.x) {
     aabft_block_report *r = a.rep + blk;
     if (r->status != AABFT_BLK_SINGLE) continue;
-    const int64_t I = blk / nJ, J = blk % nJ, i = r->row, j = r->col;
-    // c_ij <- Ccol[I][j] - sum_{i' != i} c_i'j  (reading R15; double, ascending i')
-    double v = (double)static_cast<const T *>(a.Ccol)[I * a.ld_ccol + j];
-    for (int64_t ii = I * bs; ii < I * bs + bs; ++ii)
-      if (ii != i) v = v - (double)C[ii * a.ldc + j];
-    C[i * a.ldc + j] = (T)v;
-    // re-verify row i
-    double ref = 0.0;
-    for (int64_t jj = J * bs; jj < J * bs + bs; ++jj) ref = ref + (double)C[i * a.ldc + jj];
-    const double d = ref - (double)static_cast<const T *>(a.Crow)[i * a.ld_crow + J];
-    const Bound b = row_bound<EXT, P>(a, bp, i, J);
-    if (a.Rcol) {
-      // fused check: the epilogue reference sums still describe the faulty element; refresh
-      // the two that pass through (i, j) from the corrected C so a later aabft_check of the
-      // same product sees the corrected state (ascending order, double)
-      double rc = 0.0;
-      for (int64_t ii = I * bs; ii < I * bs + bs; ++ii) rc = rc + (double)C[ii * a.ldc + j];
-      const_cast<double *>(a.Rcol)[I * a.N + j] = rc;
-      const_cast<double *>(a.Rrow)[i * nJ + J] = ref;
-    }
+    const uint8_t st = correct_block<T, P, EXT>(a, bp, C, blk, r->row, r->col);
+    r->status = st;
     unsigned long long *n = reinterpret_cast<unsigned long long *>(a.cnt->n);
-    if (fabs(d) <= b.eps) {
-      r->status = AABFT_BLK_CORRECTED;
-      atomicAdd(&n[2], 1ull);
-    } else {
-      r->status = AABFT_BLK_UNCORRECTABLE;
-      atomicAdd(&n[4], 1ull);
-    }
+    atomicAdd(&n[st == AABFT_BLK_CORRECTED ? 2 : 4], 1ull);
   }
 }
 
@@ -567,6 +620,8 @@ CheckArgs make_args(const aabft_config *cfg, const aabft_encoded *enc, const aab
   a.col_parts = a.row_parts = 1;
   a.eps_col = a.eps_row = nullptr;
   a.eps_fixed = 0.0;
+  a.acc = nullptr;
+  a.correct = (cfg->flags & AABFT_FLAG_CHECK_CORRECTS) ? 1 : 0;
   if (a.Rcol && cfg->dtype == AABFT_F64) {  // the FP32 epilogue always completes its sums
     a.col_parts = gemm_f64_fused_parts(cfg->bs, &a.row_parts);
     double *rc2, *rr2;
@@ -690,10 +745,11 @@ aabft_status launch_bound_elements(const aabft_config *cfg, const aabft_encoded 
 
 aabft_status launch_check(const aabft_config *cfg, const aabft_encoded *enc,
                           const aabft_product *prod, aabft_block_report *rep, aabft_counts *cnt,
-                          void *gemm_ws, cudaStream_t st) {
+                          void *gemm_ws, unsigned long long *acc, cudaStream_t st) {
   const BoundParams bp = make_bound_params(cfg);
-  const CheckArgs a = make_args(cfg, enc, prod, rep, cnt, gemm_ws);
-  if (cudaMemsetAsync(cnt, 0, sizeof(aabft_counts), st) != cudaSuccess)
+  CheckArgs a = make_args(cfg, enc, prod, rep, cnt, gemm_ws);
+  a.acc = acc;
+  if (!acc && cudaMemsetAsync(cnt, 0, sizeof(aabft_counts), st) != cudaSuccess)
     return check_launch("aabft_check memset");
   if (cfg->dtype == AABFT_F64) {
     AABFT_P_SWITCH(cfg->p, return (run_check<double, PP>(cfg, a, bp, st)));
@@ -724,13 +780,14 @@ aabft_status launch_correct(const aabft_config *cfg, const aabft_encoded *enc,
 aabft_status launch_check_ext(const aabft_config *cfg, const aabft_product *prod,
                               const double *eps_col, const double *eps_row, double eps_fixed,
                               aabft_block_report *rep, aabft_counts *cnt, void *gemm_ws,
-                              cudaStream_t st) {
+                              unsigned long long *acc, cudaStream_t st) {
   const BoundParams bp = make_bound_params(cfg);
   CheckArgs a = make_args(cfg, nullptr, prod, rep, cnt, gemm_ws);
   a.eps_col = eps_col;
   a.eps_row = eps_row;
   a.eps_fixed = eps_fixed;
-  if (cudaMemsetAsync(cnt, 0, sizeof(aabft_counts), st) != cudaSuccess)
+  a.acc = acc;
+  if (!acc && cudaMemsetAsync(cnt, 0, sizeof(aabft_counts), st) != cudaSuccess)
     return check_launch("aabft_check_ext memset");
   if (cfg->dtype == AABFT_F64) return run_check<double, 1, true>(cfg, a, bp, st);
   return run_check<float, 1, true>(cfg, a, bp, st);

@@ -52,10 +52,12 @@ aabft_status launch_encode(const aabft_config *cfg, const void *A, int64_t lda, 
                            int64_t ldb, const aabft_encoded *out, void *ws, cudaStream_t st);
 aabft_status launch_bound(const aabft_config *cfg, const aabft_encoded *enc, double *eps_col,
                           double *sig_col, double *eps_row, double *sig_row, cudaStream_t st);
+// check_acc (protected product): the check accumulator the kernel zeroes (see launch_check)
 aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda,
                              const void *B, int64_t ldb, const aabft_encoded *enc,
                              const aabft_product *out, const aabft_fault *faults,
-                             int32_t nfaults, bool plain, void *ws, cudaStream_t st);
+                             int32_t nfaults, bool plain, void *ws,
+                             unsigned long long *check_acc, cudaStream_t st);
 size_t encode_ws_bytes(const aabft_config *cfg);
 // AABFT_FLAG_OVERLAP_ENCODE honoured by aabft_encode (FP64, 16 <= bs <= 64, p <= 4)
 bool encode_overlap_ok(const aabft_config *cfg);
@@ -72,7 +74,8 @@ int gemm_f64_fused_parts(int bs, int *row_parts);  // returns column parts
 aabft_status launch_gemm_f32(const aabft_config *cfg, const void *A, int64_t lda,
                              const void *B, int64_t ldb, const aabft_encoded *enc,
                              const aabft_product *out, const aabft_fault *faults,
-                             int32_t nfaults, bool plain, cudaStream_t st);
+                             int32_t nfaults, bool plain, unsigned long long *check_acc,
+                             cudaStream_t st);
 aabft_status launch_bound_elements(const aabft_config *cfg, const aabft_encoded *enc,
                                    const int64_t *rows, const int64_t *cols, int64_t n,
                                    double *sig, double *eps, cudaStream_t st);
@@ -80,9 +83,11 @@ aabft_status launch_checksum_errors(const aabft_config *cfg, const void *A, int6
                                     const void *B, int64_t ldb, const aabft_encoded *enc,
                                     const aabft_product *prod, double *err_col, double *err_row,
                                     cudaStream_t st);
+// acc: the workspace's check accumulator (10 words, zeroed by aabft_gemm) or NULL (memset cnt)
 aabft_status launch_check(const aabft_config *cfg, const aabft_encoded *enc,
                           const aabft_product *prod, aabft_block_report *rep,
-                          aabft_counts *cnt, void *gemm_ws, cudaStream_t st);
+                          aabft_counts *cnt, void *gemm_ws, unsigned long long *acc,
+                          cudaStream_t st);
 aabft_status launch_correct(const aabft_config *cfg, const aabft_encoded *enc,
                             const aabft_product *prod, aabft_block_report *rep,
                             aabft_counts *cnt, cudaStream_t st);
@@ -90,7 +95,7 @@ aabft_status launch_correct(const aabft_config *cfg, const aabft_encoded *enc,
 aabft_status launch_check_ext(const aabft_config *cfg, const aabft_product *prod,
                               const double *eps_col, const double *eps_row, double eps_fixed,
                               aabft_block_report *rep, aabft_counts *cnt, void *gemm_ws,
-                              cudaStream_t st);
+                              unsigned long long *acc, cudaStream_t st);
 aabft_status launch_correct_ext(const aabft_config *cfg, const aabft_product *prod,
                                 const double *eps_row, double eps_fixed, aabft_block_report *rep,
                                 aabft_counts *cnt, cudaStream_t st);

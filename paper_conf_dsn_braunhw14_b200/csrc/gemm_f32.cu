@@ -65,6 +65,7 @@ struct SgemmArgs {
   double *Rcol;  // fused reference sums (NULL = unfused): (M/bs) x N, M x (N/bs)
   double *Rrow;
   int bs;
+  unsigned long long *check_acc;  // the following aabft_check's counter accumulator: zeroed
 };
 
 __device__ __forceinline__ float xor_bits(float v, uint64_t m) {
@@ -96,6 +97,7 @@ __global__ void __launch_bounds__(THREADS, AABFT_F32_MINB) gemm_f32_kernel(const
   aabft_fault *s_f = reinterpret_cast<aabft_fault *>(smem32 + (RING32 > TILE32 ? RING32 : TILE32));
   __shared__ int s_nf;
 
+  if (blockIdx.x == 0 && threadIdx.x < 10 && args.check_acc) args.check_acc[threadIdx.x] = 0ull;
   int64_t bid = blockIdx.x;
   int type, tm, tn;
   if (bid < args.n0) {
@@ -349,9 +351,10 @@ __global__ void __launch_bounds__(THREADS, AABFT_F32_MINB) gemm_f32_kernel(const
 aabft_status launch_gemm_f32(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
                              int64_t ldb, const aabft_encoded *enc, const aabft_product *out,
                              const aabft_fault *faults, int32_t nfaults, bool plain,
-                             cudaStream_t st) {
+                             unsigned long long *check_acc, cudaStream_t st) {
   const int64_t M = cfg->M, N = cfg->N, K = cfg->K, bs = cfg->bs;
   SgemmArgs a{};
+  a.check_acc = plain ? nullptr : check_acc;
   a.A = static_cast<const float *>(A); a.lda = lda;
   a.B = static_cast<const float *>(B); a.ldb = ldb;
   a.Acs = plain ? nullptr : static_cast<const float *>(enc->Acs);

@@ -128,6 +128,7 @@ struct GemmArgs {
   int *tp_i;
   int *tp_flags;                      // [kMaxCtas]
   int b3d, bcs3d;                     // B / Bcs tiles as ONE 3-D TMA box (8 cols x 16 k x 8 groups)
+  unsigned long long *check_acc;      // the following aabft_check's counter accumulator: zeroed
 };
 
 struct Tile {
@@ -438,6 +439,11 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
 #ifdef AABFT_OV_PROBE
   if (threadIdx.x == 0) atomicMin(&g_gemm_probe[0], gemm_gtime());
 #endif
+  if (threadIdx.x == 0 && blockIdx.x == 0 && args.check_acc) {
+    // the check of this product accumulates its counters here (no memset between the kernels)
+#pragma unroll
+    for (int w = 0; w < 10; ++w) args.check_acc[w] = 0ull;
+  }
   if (threadIdx.x == 0) {
     for (int s = 0; s < STAGES; ++s) {
       mbar_init(&full[s], 1);
@@ -954,7 +960,7 @@ void gemm_f64_red_ptrs(const aabft_config *cfg, void *ws, double **rcol2, double
 aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda, const void *B,
                              int64_t ldb, const aabft_encoded *enc, const aabft_product *out,
                              const aabft_fault *faults, int32_t nfaults, bool plain, void *ws,
-                             cudaStream_t st) {
+                             unsigned long long *check_acc, cudaStream_t st) {
   // per-device one-time setup (function attributes belong to the device's context); a racing
   // first call computes the same value twice, which is benign
   static std::atomic<int> max_ctas_dev[64];
@@ -1030,6 +1036,7 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
   a.topB_i = tp ? enc->topB_idx : nullptr;
   a.faults = faults;
   a.nfaults = faults ? nfaults : 0;
+  a.check_acc = plain ? nullptr : check_acc;
   a.bs = (int)bs;
   const bool fused = !plain && out->Rcol && out->Rrow && bs <= TILE;
   a.Rcol = fused ? out->Rcol : nullptr;

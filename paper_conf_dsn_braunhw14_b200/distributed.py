@@ -9,7 +9,7 @@ outside the step).  Every BS x BS block's encode, bound, check and correction is
   and checksum columns, in the sm_100a encode kernel -- and one all-gather gives every rank
   the full Bcs and top-p tables of B (ShardedProtectedGemm), instead of every rank re-reading
   all of B;
-* after aabft_correct, the fault counters: SUM over the int64 counters and MAX over
+* after the check (which corrects in the same kernel), the fault counters: SUM over the int64 counters and MAX over
   max |d|/eps, so every rank learns whether any block anywhere was corrected or is
   uncorrectable.
 Collectives are NCCL over NVLink on the GPU box; the gloo backend (CPU staging) lets the same
@@ -140,9 +140,7 @@ class ShardedProtectedGemm:
         nf = 0 if fbuf is None else fbuf.numel() // 48
         self.encode(A_local, B, stream)
         pl.gemm(A_local, B, fbuf, nf, stream)
-        pl.check(stream)
-        if correct:
-            pl.correct(stream)
+        pl.check(stream, correct=correct)  # correction inside the check kernel
         reduce_counts(pl.counts, self.group)
         return pl.result()
 
