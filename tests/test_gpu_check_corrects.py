@@ -48,10 +48,10 @@ def faults_for(M, N, bs, n, seed):
 CASES = [
     (torch.float64, 512, 640, 300, 64, 2, True),
     (torch.float64, 512, 640, 300, 64, 2, False),
-    (torch.float64, 256, 256, 129, 32, 3, True),
+    (torch.float64, 256, 256, 130, 32, 3, True),
     (torch.float64, 256, 512, 200, 128, 2, False),   # bs > 64: the streaming check
     (torch.float32, 512, 512, 256, 64, 2, True),
-    (torch.float32, 256, 256, 300, 256, 2, False),
+    (torch.float32, 768, 768, 300, 256, 2, False),   # 3 x 3 blocks of 256
 ]
 
 

@@ -48,13 +48,16 @@ OVERLAP_SHAPES = [
 ]
 
 
+@pytest.mark.parametrize("overlap", [True, False])
 @pytest.mark.parametrize("shape", OVERLAP_SHAPES)
-def test_overlap_encode_bit_exact(P, orc, shape):
+def test_overlap_encode_bit_exact(P, orc, shape, overlap):
+    """overlap=True: the co-resident encode grid; overlap=False: the default chunked kernels
+    (encode_ab + topp_reduce) at the same ragged shapes."""
     M, N, K, bs, p = shape
     A = synth.generate("uniform", M, K, seed=11, matrix_id=0)
     B = synth.generate("wide", K, N, seed=11, matrix_id=1)
-    plan = P.ProtectedGemm(M, N, K, dtype=torch.float64, bs=bs, p=p, overlap=True)
-    assert plan.overlap
+    plan = P.ProtectedGemm(M, N, K, dtype=torch.float64, bs=bs, p=p, overlap=overlap)
+    assert plan.overlap == overlap
     plan.topA_val.fill_(-7.0)
     plan.topB_idx.fill_(-7)
     plan.encode(to_dev(A), to_dev(B))
@@ -68,13 +71,14 @@ def test_overlap_encode_bit_exact(P, orc, shape):
     assert np.array_equal(host(plan.topB_idx), enc["topB"][1])
 
 
+@pytest.mark.parametrize("overlap", [True, False])
 @pytest.mark.parametrize("bs", [16, 32, 64])
-def test_overlap_encode_ties_integer_data(P, orc, bs):
+def test_overlap_encode_ties_integer_data(P, orc, bs, overlap):
     """Many equal |values|: lowest index wins in every merge of the complete-vector units."""
     M, N, K, p = 128, 192, 333, 4
     A = synth.generate("integer", M, K, seed=12, matrix_id=0, q=2)
     B = synth.generate("integer", K, N, seed=12, matrix_id=1, q=2)
-    plan = P.ProtectedGemm(M, N, K, dtype=torch.float64, bs=bs, p=p, overlap=True)
+    plan = P.ProtectedGemm(M, N, K, dtype=torch.float64, bs=bs, p=p, overlap=overlap)
     plan.encode(to_dev(A), to_dev(B))
     torch.cuda.synchronize()
     enc = orc.encode(A, B, bs, p)
