@@ -78,7 +78,10 @@ constexpr int CTAS_PER_SM = AABFT_F64_CTAS;  // 15 / 18 warps per SM (128 / <= 1
 // BS = 64 on a 64 x 64 tile of 2 x 2 warps: the block is the CTA tile, and the epilogue
 // completes its column / row reference sums inside the CTA (shared memory, one barrier) --
 // otherwise a block larger than a warp tile leaves per-warp "parts" in the workspace
-constexpr bool kCtaSums = TM == 64 && TN == 64 && WTN == 32;
+#ifndef AABFT_F64_CTA_SUMS
+#define AABFT_F64_CTA_SUMS 1
+#endif
+constexpr bool kCtaSums = AABFT_F64_CTA_SUMS && TM == 64 && TN == 64 && WTN == 32;
 constexpr int COL_PARTS = kCtaSums ? 1 : 2;           // fused column sums of a BS = 64 block
 constexpr int ROW_PARTS = kCtaSums ? 1 : 64 / WTN;    // fused row sums of a BS = 64 block
 constexpr int A_BYTES = TILE * BK * 8;      // 8 KiB
