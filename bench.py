@@ -357,6 +357,8 @@ def main():
 
     # per-stage device times of one protected step, and Table I's comparators (NEXT-3)
     stages = stage_times(plan, A, B, stream, dev, args.steps)
+    stage_roofs = stage_rooflines(stages, m_local, N, K, bs, P_TOPP,
+                                  8 if wl["dtype"] == "f64" else 4, plan.fused)
     table1 = None
     unfused = None
     if world == 1:
@@ -430,7 +432,8 @@ def main():
                          "algorithmic_flops_per_launch": aug_flops,
                          "avg_launch_ms": gemm_avg,
                          "share_of_step": gemm_avg / (ms / args.steps)},
-            "stages_ms": stages, "table1": table1, "unfused_check": unfused,
+            "stages_ms": stages, "stage_rooflines": stage_roofs, "table1": table1,
+            "unfused_check": unfused,
             "e2e": e2e, "gpu_launches": launches, "cpu_baseline": cpu,
             "clocks": clk.summary(),
         }
@@ -469,6 +472,35 @@ def measure_traffic(wl, m_local, N, K, bs):
     if seen != 2:
         return None, "ncu probe: metrics not found (" + (r.stderr or r.stdout)[-160:] + ")"
     return total, f"ncu dram__bytes_read+write.sum, one {kern} launch, same shape, this run"
+
+
+def hbm_peak():
+    """Measured HBM GB/s of this pod (MEASURED_PEAKS.json, driver-written), else the profiling
+    guide's fallback figure."""
+    try:
+        with open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "MEASURED_PEAKS.json")) as f:
+            return float(json.load(f)["hbm_gbs"]), "MEASURED_PEAKS.json hbm_gbs"
+    except (OSError, KeyError, ValueError):
+        return 7700.0, "nominal HBM3e fallback (no MEASURED_PEAKS.json)"
+
+
+def stage_rooflines(stages, M, N, K, bs, p, w, fused):
+    """HBM roofline of the encode and check stages (north_star: achieved HBM GB/s for encode
+    and check).  ALGORITHMIC bytes: encode reads A and B and writes Acs, Bcs and the top-p
+    tables; the fused check reads the epilogue reference sums (double), the carried checksums,
+    every vector's top-p list once and writes the block reports; the unfused check also reads C."""
+    peak, src = hbm_peak()
+    nI, nJ = M // bs, N // bs
+    vecs = M + nI + N + nJ
+    enc = (M * K + K * N) * w + (nI * K + K * nJ) * w + vecs * p * 12
+    chk = (nI * N + M * nJ) * (8 + w) + vecs * p * 12 + nI * nJ * 20 + (0 if fused else M * N * w)
+    out = {"peak_gbs": peak, "peak_source": src}
+    for name, b in (("encode", enc), ("check", chk)):
+        ms = stages.get(name)
+        if ms:
+            gbs = b / (ms * 1e-3) / 1e9
+            out[name] = {"bytes": b, "ms": ms, "achieved_gbs": gbs, "frac": gbs / peak}
+    return out
 
 
 def stage_times(plan, A, B, stream, dev, steps):

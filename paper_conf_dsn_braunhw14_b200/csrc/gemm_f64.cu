@@ -1018,7 +1018,10 @@ aabft_status launch_gemm_f64(const aabft_config *cfg, const void *A, int64_t lda
   const int64_t total = ntiles * nk;
   // AABFT_FLAG_GEMM_HALF_GRID: half the persistent grid, so two launches can share the GPU
   const int cap = (cfg->flags & AABFT_FLAG_GEMM_HALF_GRID) ? std::max(1, max_ctas / 2) : max_ctas;
-  const int grid = (int)std::min<int64_t>(cap, total);
+  // small problems: at least kMinIters k-tiles per CTA, so a split tile has few contributors
+  // (the owner adds their partials one after another: at 128^3 every tile was split 8 ways)
+  constexpr int64_t kMinIters = 4;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(cap, std::max<int64_t>(ntiles, total / kMinIters)));
   // full data-parallel waves, keeping at least ~1/2 wave of tiles for the stream-K tail so
   // every CTA's k-slice stays long enough to amortise its fixup
   int waves = (int)(ntiles / grid);
