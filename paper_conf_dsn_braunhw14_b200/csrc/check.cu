@@ -265,10 +265,11 @@ __device__ __forceinline__ uint8_t maybe_correct(const CheckArgs &a, const Bound
 // CTA counters (s_n[8], s_mr: float bits) -> device totals.  With a workspace accumulator the
 // CTAs add into it and the LAST CTA (ticket) moves the totals into `cnt` and re-arms the
 // accumulator (threadfence-reduction pattern); otherwise straight atomics into the zeroed cnt.
-__device__ __forceinline__ void publish_counts(const CheckArgs &a, const unsigned long long *s_n,
-                                               unsigned s_mr, int tid) {
+template <typename CT>
+__device__ __forceinline__ void publish_counts(const CheckArgs &a, const CT *s_n, unsigned s_mr,
+                                               int tid) {
   unsigned long long *dst = a.acc ? a.acc : reinterpret_cast<unsigned long long *>(a.cnt->n);
-  if (tid < 8 && s_n[tid]) atomicAdd(dst + tid, s_n[tid]);
+  if (tid < 8 && s_n[tid]) atomicAdd(dst + tid, (unsigned long long)s_n[tid]);
   if (tid == 8 && s_mr) atomicMax(dst + 8, (unsigned long long)__double_as_longlong((double)__uint_as_float(s_mr)));
   if (!a.acc) return;
   __shared__ bool s_last;
@@ -307,19 +308,26 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
   constexpr int MAXJB = kFusedThreads / 8;  // bs >= 8
   __shared__ int s_nr[MAXJB], s_nc[MAXJB], s_row[MAXJB], s_col[MAXJB], s_worst[MAXJB];
   __shared__ unsigned s_rmax[MAXJB];  // float bits (non-negative: integer order = value order)
-  __shared__ unsigned long long s_n[8];
+  __shared__ unsigned s_n[8];  // 32-bit: native shared atomics
   __shared__ unsigned s_mr;
   const int tid = threadIdx.x, lane = tid & 31;
   const int bs = a.bs, JB = kFusedThreads / bs;
+  const int lbs = __ffs(bs) - 1, ljb = __ffs(JB) - 1;  // bs, JB are powers of two
   const int64_t nJ = a.N / bs;
-  if (tid < 8) s_n[tid] = 0ull;
+  if (tid < 8) s_n[tid] = 0u;
   if (tid == 8) s_mr = 0u;
   unsigned my_n[5] = {0, 0, 0, 0, 0};  // blocks, clean, corrected, checksum-only, uncorrectable
   unsigned cls0 = 0, cls1 = 0, cls2 = 0;  // checks per class (registers, not an indexed array)
   float mr = 0.f;
   const int cseg = bs < 32 ? bs : 32;  // lanes sharing one block among the column checks
+  // unit u = I * ngrp + g, advanced by gridDim.x with a carry (no division in the loop)
+  const unsigned du = gridDim.x / (unsigned)ngrp, dg = gridDim.x % (unsigned)ngrp;
+  unsigned uI = blockIdx.x / (unsigned)ngrp, ug = blockIdx.x % (unsigned)ngrp;
   for (int64_t u = blockIdx.x; u < nunits; u += gridDim.x) {
-    const int64_t I = u / ngrp, J0 = (u % ngrp) * JB;
+    const int64_t I = uI, J0 = (int64_t)ug << ljb;
+    uI += du;
+    ug += dg;
+    if (ug >= (unsigned)ngrp) { ug -= (unsigned)ngrp; ++uI; }
     if (tid < JB) {
       s_nr[tid] = 0; s_nc[tid] = 0; s_row[tid] = -1; s_col[tid] = -1; s_worst[tid] = 0;
       s_rmax[tid] = 0u;
@@ -327,10 +335,10 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
     __syncthreads();
     // Both checks' operands are gathered first (every load of the thread in flight together),
     // then the part sums are written back, then classified.
-    const int Jc = tid / bs;                                   // column check: block of j
-    const int64_t j = J0 * bs + tid;
-    const int ii = tid / JB, Jr = tid - (tid / JB) * JB;      // row check: (i, J)
-    const int64_t J = J0 + Jr, i = I * bs + ii;
+    const int Jc = tid >> lbs;                                 // column check: block of j
+    const int64_t j = (J0 << lbs) + tid;
+    const int ii = tid >> ljb, Jr = tid & (JB - 1);            // row check: (i, J)
+    const int64_t J = J0 + Jr, i = (I << lbs) + ii;
     const bool hc = j < a.N, hr = J < nJ;
     double refc = 0.0, carc = 0.0, refr = 0.0, carr = 0.0, rc2 = 0.0, rp[7] = {};  // row_parts <= 64 / 8
     Bound bc{0.0, 0.0}, brw{0.0, 0.0};
@@ -377,7 +385,9 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
       if (cseg == 32) {
         rb = __reduce_max_sync(0xffffffffu, rb);
       } else {
-        for (int m = 1; m < cseg; m <<= 1) rb = max(rb, __shfl_xor_sync(0xffffffffu, rb, m));
+#pragma unroll
+        for (int m = 1; m < 32; m <<= 1)
+          if (m < cseg) rb = max(rb, __shfl_xor_sync(0xffffffffu, rb, m));  // uniform condition
       }
       if ((lane & (cseg - 1)) == 0 && rb) atomicMax(&s_rmax[Jc], rb);
     }
@@ -394,7 +404,9 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
         r = (float)ratio_fast(d, brw.eps);
       }
       unsigned rb = __float_as_uint(r);
-      for (int m = JB; m < 32; m <<= 1) rb = max(rb, __shfl_xor_sync(0xffffffffu, rb, m));
+#pragma unroll
+      for (int m = 1; m < 32; m <<= 1)
+        if (m >= JB) rb = max(rb, __shfl_xor_sync(0xffffffffu, rb, m));  // uniform condition
       if (lane < JB && rb) atomicMax(&s_rmax[Jr], rb);
     }
     __syncthreads();
@@ -447,7 +459,7 @@ __global__ void __launch_bounds__(kFusedThreads) check_fused_kernel(CheckArgs a,
   if (lane == 0) {
 #pragma unroll
     for (int c = 0; c < 8; ++c)
-      if (wn[c]) atomicAdd(&s_n[c], (unsigned long long)wn[c]);
+      if (wn[c]) atomicAdd(&s_n[c], wn[c]);
     if (wmr) atomicMax(&s_mr, wmr);
   }
   __syncthreads();
