@@ -61,6 +61,9 @@ constexpr bool B16 = AABFT_F64_B16 != 0;
 #ifndef AABFT_F64_L2PROMO
 #define AABFT_F64_L2PROMO CU_TENSOR_MAP_L2_PROMOTION_L2_128B
 #endif
+#ifndef AABFT_F64_C_STREAM
+#define AABFT_F64_C_STREAM 0
+#endif
 #ifndef AABFT_F64_NT
 #define AABFT_F64_NT 4
 #endif
@@ -372,6 +375,21 @@ __device__ __forceinline__ void scan_job(const GemmArgs &a, const uint8_t *smem,
   }
 }
 
+#ifndef AABFT_F64_EVICT_LAST
+#define AABFT_F64_EVICT_LAST 0
+#endif
+// TMA load with an L2 evict-last hint (operand panels are re-read by many CTAs)
+__device__ __forceinline__ void tma_load_2d_el(void *smem_dst, const CUtensorMap *tm, uint64_t *bar,
+                                               int c0, int c1) {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1, {%3, %4}], [%2], %5;" ::"r"(smem_u32(smem_dst)),
+      "l"(reinterpret_cast<uint64_t>(tm)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "l"(pol)
+      : "memory");
+}
+
 // one stage of a job: expect the bytes, then the A box and the B tile (one 3-D box, or 2-D
 // boxes of 8 / 16 columns), all from the calling thread
 __device__ __forceinline__ void issue_stage(const GemmArgs &a, const CUtensorMap *tmA,
@@ -386,12 +404,22 @@ __device__ __forceinline__ void issue_stage(const GemmArgs &a, const CUtensorMap
     tma_load_3d(sa + A_BYTES, mb, bar, 0, k, tl.n0 / 8);
   } else if (B16) {
 #pragma unroll
-    for (int b = 0; b < TN / 16; ++b) tma_load_2d(sa + A_BYTES + b * 2048, mb, bar, tl.n0 + b * 16, k);
+    for (int b = 0; b < TN / 16; ++b) {
+#if AABFT_F64_EVICT_LAST
+      tma_load_2d_el(sa + A_BYTES + b * 2048, mb, bar, tl.n0 + b * 16, k);
+#else
+      tma_load_2d(sa + A_BYTES + b * 2048, mb, bar, tl.n0 + b * 16, k);
+#endif
+    }
   } else {
 #pragma unroll
     for (int b = 0; b < TN / 8; ++b) tma_load_2d(sa + A_BYTES + b * 1024, mb, bar, tl.n0 + b * 8, k);
   }
+#if AABFT_F64_EVICT_LAST
+  tma_load_2d_el(sa, tl.type == 1 ? tmAcs : tmA, bar, k, tl.m0);
+#else
   tma_load_2d(sa, tl.type == 1 ? tmAcs : tmA, bar, k, tl.m0);
+#endif
 }
 
 #ifdef AABFT_OV_PROBE
@@ -839,7 +867,11 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
           double *p = out + r * ld + c;
           const double v0 = acc[mt][nt][h * 2], v1 = acc[mt][nt][h * 2 + 1];
           if (c + 1 < cols_valid && vec_ok) {
+#if AABFT_F64_C_STREAM
+            __stcs(reinterpret_cast<double2 *>(p), make_double2(v0, v1));  // evict-first: keep L2 for operands
+#else
             *reinterpret_cast<double2 *>(p) = make_double2(v0, v1);
+#endif
           } else {
             if (c < cols_valid) p[0] = v0;
             if (c + 1 < cols_valid) p[1] = v1;
