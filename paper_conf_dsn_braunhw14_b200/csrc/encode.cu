@@ -395,7 +395,10 @@ __global__ void __launch_bounds__(NC) encode_b_kernel(const T *__restrict__ B, i
 // then the A units; one shared buffer serves whichever body the CTA runs.  Saves a launch
 // boundary and lets the A units fill the machine while B's last units finish.
 template <typename T, int P, bool TOPP>
-__global__ void __launch_bounds__(128) encode_ab_kernel(
+#ifndef AABFT_ENC_MINB
+#define AABFT_ENC_MINB 1
+#endif
+__global__ void __launch_bounds__(128, AABFT_ENC_MINB) encode_ab_kernel(
     const T *__restrict__ A, int64_t lda, int64_t M, int64_t K, int bs, T *__restrict__ Acs,
     int64_t ld_acs, double *__restrict__ pva, int *__restrict__ pia, int ncha,
     const T *__restrict__ B, int64_t ldb, int64_t N, T *__restrict__ Bcs, int64_t ld_bcs,

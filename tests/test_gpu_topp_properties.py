@@ -1,0 +1,55 @@
+"""Full-size top-p properties (BASELINE configs[1] and [2] shapes), checked with a library sort.
+
+Alg 1 selects, per row of A / column of B and per checksum row / column, the p
+largest |values|; reading R13 fixes the order (value descending, ties to the lowest index).  At
+full size the sequential oracle is too slow to run over every vector, but the selection has a
+plain definition: the first p entries of a STABLE descending sort of |vector|.  torch.sort (a
+library primitive, independent of this repo's kernels) gives that permutation, so every index,
+every value and the tie order are compared for every vector -- data and checksum vectors -- and
+the indices of each list are distinct by construction of the comparison.
+"""
+import numpy as np
+import pytest
+
+import synth
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def P():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_dsn_braunhw14_b200 import api
+    return api
+
+
+def first_p_stable(X, p):
+    """(values, indices) of the first p entries of a stable descending sort of |X| per row."""
+    v, i = torch.sort(X.abs().to(torch.float64), dim=1, descending=True, stable=True)
+    return v[:, :p], i[:, :p].to(torch.int32)
+
+
+@pytest.mark.parametrize("case", [
+    ("f64", 4096, 4096, 4096, 64, 2, "uniform"),     # configs[1]
+    ("f32", 8192, 8192, 8192, 64, 2, "wide"),        # configs[2]
+    ("f64", 4096, 4096, 4096, 64, 2, "integer"),     # many exact ties
+])
+def test_topp_full_size_equals_stable_sort(P, case):
+    dt, M, N, K, bs, p, recipe = case
+    npdt = np.float64 if dt == "f64" else np.float32
+    tdt = torch.float64 if dt == "f64" else torch.float32
+    kw = dict(q=3) if recipe == "integer" else {}
+    A = torch.from_numpy(synth.generate(recipe, M, K, seed=31, matrix_id=0, dtype=npdt, **kw)).cuda()
+    B = torch.from_numpy(synth.generate(recipe, K, N, seed=31, matrix_id=1, dtype=npdt, **kw)).cuda()
+    plan = P.ProtectedGemm(M, N, K, dtype=tdt, bs=bs, p=p)
+    plan.encode(A, B)
+    torch.cuda.synchronize()
+    rowsA = torch.cat([A, plan.Acs], dim=0)          # data rows, then checksum rows
+    colsB = torch.cat([B.t(), plan.Bcs.t()], dim=0)  # data columns, then checksum columns
+    for X, val, idx, name in ((rowsA, plan.topA_val, plan.topA_idx, "A"),
+                              (colsB, plan.topB_val, plan.topB_idx, "B")):
+        ev, ei = first_p_stable(X, p)
+        assert torch.equal(idx, ei), name
+        assert torch.equal(val, ev), name
