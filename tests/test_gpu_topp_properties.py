@@ -53,3 +53,32 @@ def test_topp_full_size_equals_stable_sort(P, case):
         ev, ei = first_p_stable(X, p)
         assert torch.equal(idx, ei), name
         assert torch.equal(val, ev), name
+
+
+@pytest.mark.parametrize("case", [
+    ("f64", 4096, 4096, 4096, 64),     # configs[1]
+    ("f32", 8192, 8192, 8192, 64),     # configs[2]
+])
+def test_checksums_full_size_sequential_definition(P, case):
+    """Eq 1 / Eq 2 at full size, bit for bit: Acs[I] = (((A[I*bs] + A[I*bs+1]) + ...) summed in
+    ascending order in the working precision (reading R11), written out as bs elementwise
+    library adds over all blocks at once (IEEE adds, no contraction); Bcs likewise over j."""
+    dt, M, N, K, bs = case
+    npdt = np.float64 if dt == "f64" else np.float32
+    tdt = torch.float64 if dt == "f64" else torch.float32
+    rec = "uniform" if dt == "f64" else "wide"
+    A = torch.from_numpy(synth.generate(rec, M, K, seed=32, matrix_id=0, dtype=npdt)).cuda()
+    B = torch.from_numpy(synth.generate(rec, K, N, seed=32, matrix_id=1, dtype=npdt)).cuda()
+    plan = P.ProtectedGemm(M, N, K, dtype=tdt, bs=bs, p=2)
+    plan.encode(A, B)
+    torch.cuda.synchronize()
+    Ab = A.view(M // bs, bs, K)
+    acs = Ab[:, 0].clone()
+    for r in range(1, bs):
+        acs = acs + Ab[:, r]
+    Bb = B.view(K, N // bs, bs)
+    bcs = Bb[:, :, 0].clone()
+    for c in range(1, bs):
+        bcs = bcs + Bb[:, :, c]
+    assert torch.equal(plan.Acs, acs)
+    assert torch.equal(plan.Bcs, bcs)
