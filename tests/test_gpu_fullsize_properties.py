@@ -1,4 +1,4 @@
-"""Full-size top-p properties (BASELINE configs[1] and [2] shapes), checked with a library sort.
+"""Full-size properties at BASELINE configs[1] and [2] (top-p lists, Eq 1 / Eq 2 checksums, Eq 3 product).
 
 Alg 1 selects, per row of A / column of B and per checksum row / column, the p
 largest |values|; reading R13 fixes the order (value descending, ties to the lowest index).  At
@@ -82,3 +82,30 @@ def test_checksums_full_size_sequential_definition(P, case):
         bcs = bcs + Bb[:, :, c]
     assert torch.equal(plan.Acs, acs)
     assert torch.equal(plan.Bcs, bcs)
+
+
+@pytest.mark.parametrize("case", [
+    ("f64", 4096, 4096, 4096, 64, 1e-13),   # configs[1]: north_star's FP64 bar
+    ("f32", 8192, 8192, 8192, 64, 1e-5),    # configs[2]: north_star's FP32 bar
+])
+def test_product_full_size_every_element(P, case):
+    """Eq 3 at full size, EVERY element of C, Ccol = Acs.B and Crow = A.Bcs against an FP64
+    library product of the same operands (cuBLAS via torch.matmul -- an independent
+    implementation of the plain definition), normalised by |A||B| as north_star states."""
+    dt, M, N, K, bs, tol = case
+    npdt = np.float64 if dt == "f64" else np.float32
+    tdt = torch.float64 if dt == "f64" else torch.float32
+    rec = "uniform" if dt == "f64" else "wide"
+    A = torch.from_numpy(synth.generate(rec, M, K, seed=33, matrix_id=0, dtype=npdt)).cuda()
+    B = torch.from_numpy(synth.generate(rec, K, N, seed=33, matrix_id=1, dtype=npdt)).cuda()
+    plan = P.ProtectedGemm(M, N, K, dtype=tdt, bs=bs, p=2)
+    res = plan.run(A, B)
+    torch.cuda.synchronize()
+    assert res.counts()["checks_critical"] == 0
+    A64, B64 = A.double(), B.double()
+    Acs64, Bcs64 = plan.Acs.double(), plan.Bcs.double()
+    for got, ref, den in ((res.C, A64 @ B64, A64.abs() @ B64.abs()),
+                          (res.Ccol, Acs64 @ B64, Acs64.abs() @ B64.abs()),
+                          (res.Crow, A64 @ Bcs64, A64.abs() @ Bcs64.abs())):
+        err = ((got.double() - ref).abs() / den.clamp_min(1e-300)).max().item()
+        assert err <= tol, err
