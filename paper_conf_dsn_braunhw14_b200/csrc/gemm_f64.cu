@@ -61,6 +61,9 @@ constexpr bool B16 = AABFT_F64_B16 != 0;
 #ifndef AABFT_F64_L2PROMO
 #define AABFT_F64_L2PROMO CU_TENSOR_MAP_L2_PROMOTION_L2_128B
 #endif
+#ifndef AABFT_F64_KROT
+#define AABFT_F64_KROT 0
+#endif
 #ifndef AABFT_F64_C_STREAM
 #define AABFT_F64_C_STREAM 0
 #endif
@@ -513,7 +516,14 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
       const int s = jn % STAGES;
       if (jn >= STAGES) mbar_wait(&empty[s], (uint32_t)(((jn / STAGES) & 1) ^ 1));
       uint8_t *sa = smem + s * STAGE_BYTES;
-      const int k = kt * BK;
+      // AABFT_F64_KROT (experiment): the CTAs sharing an SM start their data-parallel tiles at
+      // k offsets 0, nk/3, 2nk/3 so their k-tile boundaries do not coincide
+      int kphys = kt;
+      if (AABFT_F64_KROT && !FAULTS && TP == 0 && jn < args.waves * args.nk) {
+        const int rot = (int)(((long long)blockIdx.x * 3) / gridDim.x) * (args.nk / 3);
+        kphys = (kt + rot) % args.nk;
+      }
+      const int k = kphys * BK;
       if (lane == 0) {
         // checksum tiles read Acs / Bcs, which a programmatically-dependent launch may still
         // be producing: wait for the preceding grid (no-op without PDL).  Data tiles read only
