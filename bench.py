@@ -379,7 +379,8 @@ def main():
 
     # fault-injection campaign (outside the timed region): one fault per BS x BS block
     campaign = None
-    if args.campaign and rank == 0:
+    # (N = 1 only: at N > 1 the other ranks would idle in the next collective meanwhile)
+    if args.campaign and rank == 0 and world == 1:
         campaign = run_campaign(plan, A, B, wl, dev, ndt)
 
     # end-to-end through the C ABI with HOST buffers (pinned), copies inside the timed region
