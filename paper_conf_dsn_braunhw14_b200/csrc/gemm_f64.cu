@@ -61,6 +61,9 @@ constexpr bool B16 = AABFT_F64_B16 != 0;
 #ifndef AABFT_F64_L2PROMO
 #define AABFT_F64_L2PROMO CU_TENSOR_MAP_L2_PROMOTION_L2_128B
 #endif
+#ifndef AABFT_F64_EARLY_RELEASE
+#define AABFT_F64_EARLY_RELEASE 0
+#endif
 #ifndef AABFT_F64_KROT
 #define AABFT_F64_KROT 0
 #endif
@@ -660,6 +663,12 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
       for (int ks = 0; ks < BK / 4; ++ks) {
         if (ks + 1 < BK / 4) {
           load(st, (ks + 1) & 1, ks + 1);
+#if AABFT_F64_EARLY_RELEASE
+          if (ks + 2 == BK / 4) {  // the stage's last fragments are loaded: release it now
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[s]);
+          }
+#endif
         } else if (kt + 1 < kt_end) {
           const int s1 = (j + 1) % STAGES;
           mbar_wait(&full[s1], (uint32_t)(((j + 1) / STAGES) & 1));
@@ -671,9 +680,11 @@ __global__ void __launch_bounds__(CTA_THREADS, CTAS_PER_SM)
           for (int nt = 0; nt < NT; ++nt)
             dmma(acc[mt][nt], a[ks & 1][mt][0], a[ks & 1][mt][1], b[ks & 1][nt]);
       }
+#if !AABFT_F64_EARLY_RELEASE
       // release the stage to the producer (its last fragments were consumed by the ks = 3 DMMAs)
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[s]);
+#endif
 #ifdef AABFT_F64_KSYNC
       if ((kt & (AABFT_F64_KSYNC - 1)) == 0) mma_sync_bar();  // experiment: MMA warps in lockstep
 #endif
