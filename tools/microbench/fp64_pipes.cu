@@ -91,6 +91,23 @@ __global__ void k_ffma(float* out, int iters) {
   for (int i = 0; i < NACC; ++i) s += c[i];
   out[blockIdx.x * blockDim.x + threadIdx.x] = s;
 }
+// packed fp32x2 FMA (sm_100 FFMA2) with a broadcast scalar operand -- the FP32 GEMM's form
+template<int NACC>
+__global__ void k_ffma2(float* out, int iters) {
+  const float a = threadIdx.x * 1e-3f;
+  const float2 b = make_float2(1.0f + threadIdx.x * 1e-7f, 1.0f - threadIdx.x * 1e-7f);
+  float2 c[NACC];
+  #pragma unroll
+  for (int i = 0; i < NACC; ++i) c[i] = make_float2(i, -i);
+  for (int it = 0; it < iters; ++it) {
+    #pragma unroll
+    for (int i = 0; i < NACC; ++i) c[i] = __ffma2_rn(make_float2(a, a), b, c[i]);
+  }
+  float s = 0;
+  #pragma unroll
+  for (int i = 0; i < NACC; ++i) s += c[i].x + c[i].y;
+  out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
 __global__ void k_copy(const double4* __restrict__ a, double4* __restrict__ b, size_t n) {
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) b[i] = a[i];
 }
@@ -135,6 +152,8 @@ int main() {
     report("dfma", wpb, warps * 32.0 * iters * 16 * 2, ms);
     ms = time_it([&] { k_ffma<16><<<blocks, threads>>>((float*)out, iters); }, 5);
     report("ffma", wpb, warps * 32.0 * iters * 16 * 2, ms);
+    ms = time_it([&] { k_ffma2<16><<<blocks, threads>>>((float*)out, iters); }, 5);
+    report("ffma2", wpb, warps * 32.0 * iters * 16 * 4, ms);
   }
   size_t bytes = (size_t)2 << 30; double4 *a, *b;
   CK(cudaMalloc(&a, bytes)); CK(cudaMalloc(&b, bytes)); cudaMemset(a, 0, bytes);
