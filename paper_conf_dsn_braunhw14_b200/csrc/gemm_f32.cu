@@ -37,6 +37,9 @@ constexpr int MAXF = BM * BN / 64;  // faults per tile kept in smem (one per 8x8
 constexpr int RING32 = STAGES * (BM + BN) * BK * 4;
 constexpr int TILE32 = BM * (BN + 1) * 4;  // fused-sum epilogue staging (reuses the ring)
 constexpr int SMEM32 = (RING32 > TILE32 ? RING32 : TILE32) + MAXF * (int)sizeof(aabft_fault);
+#ifndef AABFT_F32_SCALAR
+#define AABFT_F32_SCALAR 0
+#endif
 #ifndef AABFT_F32_JOUTER
 #define AABFT_F32_JOUTER 1  // measured 20.42 vs 20.61 ms at 8192^3
 #endif
@@ -261,7 +264,12 @@ __global__ void __launch_bounds__(THREADS, AABFT_F32_MINB) gemm_f32_kernel(const
 #pragma unroll
           for (int i = 0; i < 8; ++i) {
             const float av = kk == 0 ? a4[i].x : (kk == 1 ? a4[i].y : (kk == 2 ? a4[i].z : a4[i].w));
+#if AABFT_F32_SCALAR  // experiment: scalar FFMA (higher pipe ceiling, twice the instructions)
+            acc2[i][j].x = __fmaf_rn(av, bv[j].x, acc2[i][j].x);
+            acc2[i][j].y = __fmaf_rn(av, bv[j].y, acc2[i][j].y);
+#else
             acc2[i][j] = __ffma2_rn(make_float2(av, av), bv[j], acc2[i][j]);
+#endif
           }
 #else
 #pragma unroll
